@@ -1,0 +1,144 @@
+/*
+ * include/topk.h -- C ABI of the B200-native bitonic top-k library (libtopk_b200.so).
+ *
+ * The operation (PAPER.md = /root/reference/PAPER.md, "P:<line>"):
+ *   "find the top-k items, i.e., the largest or smallest ... according to some sort
+ *   order (implemented via LIMIT or ORDER BY expressions in SQL)"  -- P:16 (Abstract);
+ *   "finding the highest (or lowest) k of n tuples given a ranking function" -- P:32 (§1).
+ * The method is the paper's bitonic top-k (§3.2; Alg. 4): local
+ * sort into k-runs, merge of run pairs (keep the better element of each pair), rebuild
+ * of the resulting bitonic k-sequences, repeated until k remain.  Key types follow the
+ * paper's evaluation: float, unsigned int, double; key + value
+ * by passing the tuple id around and assembling at the end.
+ *
+ * Result definition (readings R1-R5; the paper is silent on these):
+ *   - total order: code(key) descending, then source index ascending (ties -> lowest
+ *     index).  code(): NaN (any sign/payload) ranks above +inf and all NaNs tie; -0 and
+ *     +0 tie; TOPK_SMALLEST reverses the key order but keeps "lowest index first".
+ *   - out[0..k) is best first; out_keys[j] is bit-identical to keys[out_idx[j] - base].
+ *   - any 1 <= k <= min(n, 1024) (k need not be a power of two).
+ *
+ * Conventions for every call below:
+ *   - Pointers named keys/payload/out_* and ws are DEVICE pointers (cudaMalloc or
+ *     equivalent), except in topk_select_host where h_* are HOST pointers.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     All work is enqueued asynchronously on it; nothing synchronises the host.
+ *   - Layout: 1-D contiguous arrays.  keys must be aligned to sizeof(key); 16-byte
+ *     alignment is NOT required (the unaligned head/tail is peeled).  Outputs: out_keys
+ *     [k] of the key type, out_idx [k] int64, out_payload [k] uint32; any may be NULL.
+ *   - Ownership: the caller owns every buffer; the library never allocates device
+ *     memory, never frees, and retains no pointer after the call returns.  Buffers must
+ *     stay valid until the stream reaches the enqueued work.
+ *   - Workspace: `ws` of at least topk_workspace_bytes(...) bytes, 256-byte aligned,
+ *     zero-filled before its FIRST use (topk_workspace_init); every call leaves it
+ *     zero-filled again.  One workspace must not be used by two calls concurrently;
+ *     calls with distinct workspaces are re-entrant.
+ *   - Errors: argument errors are returned synchronously and nothing is enqueued;
+ *     launch failures return TOPK_ERR_CUDA; asynchronous faults surface at the caller's
+ *     next synchronisation of `stream`.
+ */
+#ifndef TOPK_B200_H
+#define TOPK_B200_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define TOPK_ABI_VERSION 1
+#define TOPK_MAX_K 1024
+
+typedef enum {
+    TOPK_OK = 0,
+    TOPK_ERR_INVALID_ARG = 1, /* NULL input, k == 0, k > n, k > 1024, bad enum, alias  */
+    TOPK_ERR_UNSUPPORTED = 2, /* device is not sm_100 (B200)                          */
+    TOPK_ERR_WORKSPACE = 3,   /* ws NULL, too small or misaligned                      */
+    TOPK_ERR_CUDA = 4         /* a CUDA runtime call or kernel launch failed           */
+} topk_status_t;
+
+typedef enum {
+    TOPK_LARGEST = 0, /* ORDER BY key DESC LIMIT k */
+    TOPK_SMALLEST = 1 /* ORDER BY key ASC  LIMIT k */
+} topk_order_t;
+
+typedef enum { TOPK_F32 = 0, TOPK_U32 = 1, TOPK_F64 = 2 } topk_dtype_t;
+
+typedef enum {
+    /* Default.  The streaming pass keeps a key only if it can still be in the top-k
+     * (the paper's §5 "buffer filler", with the predicate "better than the
+     * current k-th best"); survivors run through local sort / merge / rebuild.
+     * Result identical to TOPK_MODE_PURE. */
+    TOPK_MODE_FILTER = 0,
+    /* The paper's pure method: every key goes through local sort, merge and rebuild
+     * (SortReducer P:179-180).  Data-independent work. */
+    TOPK_MODE_PURE = 1
+} topk_mode_t;
+
+/* Workspace bytes needed by topk_select / topk_* for (dtype, n, k) on the current
+ * device.  Returns 0 if the arguments are invalid.  O(#SM * k * 12 B), < 4 MiB. */
+size_t topk_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k);
+
+/* Zero-fill a workspace (enqueued on `stream`).  Needed once before first use. */
+topk_status_t topk_workspace_init(void* ws, size_t ws_bytes, void* stream);
+
+/* General entry point: top-k of keys[0..n) whose global row ids are base + i.
+ *   dtype     TOPK_F32 (float), TOPK_U32 (uint32_t) or TOPK_F64 (double) keys.
+ *   payload   optional uint32 column [n] gathered into out_payload; may be NULL.
+ *   base      added to every output index (shard offset, §8(e)); 0 for a plain call.
+ *   mode      TOPK_MODE_FILTER (default) or TOPK_MODE_PURE; same result.
+ *   out_idx   receives base + i of each winner (int64). */
+topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
+                          uint64_t n, uint64_t base, uint32_t k, topk_order_t order,
+                          topk_mode_t mode, void* out_keys, uint32_t* out_payload,
+                          int64_t* out_idx, void* ws, size_t ws_bytes, void* stream);
+
+/* Typed conveniences (base = 0, mode = TOPK_MODE_FILTER). */
+topk_status_t topk_f32(const float* keys, uint64_t n, uint32_t k, topk_order_t order,
+                       float* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream);
+topk_status_t topk_u32(const uint32_t* keys, uint64_t n, uint32_t k, topk_order_t order,
+                       uint32_t* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream);
+topk_status_t topk_f64(const double* keys, uint64_t n, uint32_t k, topk_order_t order,
+                       double* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream);
+/* Key + payload: "ORDER BY key DESC LIMIT k" returning the 32-bit row id column. */
+topk_status_t topk_u32_kv(const uint32_t* keys, const uint32_t* payload, uint64_t n,
+                          uint32_t k, topk_order_t order, uint32_t* out_keys,
+                          uint32_t* out_payload, int64_t* out_idx, void* ws,
+                          size_t ws_bytes, void* stream);
+topk_status_t topk_f64_kv(const double* keys, const uint32_t* payload, uint64_t n,
+                          uint32_t k, topk_order_t order, double* out_keys,
+                          uint32_t* out_payload, int64_t* out_idx, void* ws,
+                          size_t ws_bytes, void* stream);
+
+/* Global step of the partitioned top-k (§1, App. C; multi-GPU §8(e)):
+ * the exact top-k of `runs` candidate lists of `run_len` entries each, laid out
+ * back to back: cand_keys[runs*run_len] (key type), cand_idx[runs*run_len] int64
+ * global row ids (the tie-break), cand_payload optional.  Entries may be in any order;
+ * duplicated (key, idx) entries are not allowed.  1 <= k <= min(runs*run_len, 1024),
+ * runs*run_len <= 65536.  Single-CTA merge + rebuild network; ws as topk_merge_ws_bytes. */
+size_t topk_merge_workspace_bytes(topk_dtype_t dtype, uint32_t runs, uint32_t run_len,
+                                  uint32_t k);
+topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_t* cand_idx,
+                         const uint32_t* cand_payload, uint32_t runs, uint32_t run_len,
+                         uint32_t k, topk_order_t order, void* out_keys,
+                         uint32_t* out_payload, int64_t* out_idx, void* ws,
+                         size_t ws_bytes, void* stream);
+
+/* Number of kernels this library has launched in this process (for the bench's
+ * "gpu_launches" count).  Thread-safe, monotone. */
+uint64_t topk_launch_count(void);
+
+/* Static description of a status code. */
+const char* topk_status_string(topk_status_t s);
+
+/* TOPK_ABI_VERSION of the loaded library. */
+int topk_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TOPK_B200_H */

@@ -1,0 +1,131 @@
+"""B200-native bitonic top-k (Shanbhag, Pirk, Madden, SIGMOD 2018).
+
+Thin Python binding over the C ABI in ``include/topk.h`` (``libtopk_b200.so``): the
+functions below only marshal torch tensors (device memory, current stream) into the
+C calls; every step of the top-k runs in the library's sm_100a kernels.
+
+    values, indices = topk(x, k, largest=True)          # x: 1-D cuda f32/u32/f64
+    values, indices, pay = topk(x, k, payload=p)        # key + 32-bit payload
+    values, indices = merge(cand_vals, cand_idx, k)     # global step
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import _lib
+
+__all__ = ["topk", "merge", "Workspace", "launch_count", "workspace_bytes"]
+
+_DT = {torch.float32: _lib.F32, torch.uint32: _lib.U32, torch.float64: _lib.F64}
+
+
+def _dtype_code(t: torch.Tensor) -> int:
+    try:
+        return _DT[t.dtype]
+    except KeyError:
+        raise TypeError(f"unsupported key dtype {t.dtype} (float32, uint32, float64)") from None
+
+
+def _stream_ptr(device) -> ctypes.c_void_p:
+    return ctypes.c_void_p(torch.cuda.current_stream(device).cuda_stream)
+
+
+def _ptr(t):
+    return ctypes.c_void_p(t.data_ptr()) if t is not None else None
+
+
+def workspace_bytes(dtype: torch.dtype, n: int, k: int) -> int:
+    return int(_lib.load().topk_workspace_bytes(_DT[dtype], n, k))
+
+
+class Workspace:
+    """Device workspace for topk() (zero-filled once; each call leaves it zeroed).
+    Must not be shared by concurrent calls on different streams."""
+
+    def __init__(self, nbytes: int, device):
+        self.nbytes = max(256, int(nbytes))
+        self.buf = torch.zeros(self.nbytes, dtype=torch.uint8, device=device)
+
+    def ptr(self):
+        return ctypes.c_void_p(self.buf.data_ptr())
+
+
+_ws_cache: dict = {}
+
+
+def _workspace(device, nbytes: int) -> Workspace:
+    key = (device.index, torch.cuda.current_stream(device).cuda_stream)
+    ws = _ws_cache.get(key)
+    if ws is None or ws.nbytes < nbytes:
+        ws = Workspace(max(nbytes, 1 << 20), device)
+        _ws_cache[key] = ws
+    return ws
+
+
+def topk(x: torch.Tensor, k: int, largest: bool = True, payload: torch.Tensor | None = None,
+         base: int = 0, mode: str = "filter", out=None, workspace: Workspace | None = None):
+    """Exact top-k of a 1-D CUDA tensor, best first; ties -> lowest index.
+
+    Returns ``(values, indices)`` or ``(values, indices, payload_out)``; indices are
+    ``base + position`` as int64.  ``mode``: "filter" (default) or "pure" (the paper's
+    data-independent network on every key); both give identical results.
+    """
+    if not x.is_cuda or x.dim() != 1:
+        raise ValueError("topk expects a 1-D CUDA tensor (no CPU path)")
+    lib = _lib.load()
+    dt = _dtype_code(x)
+    n = x.shape[0]
+    x = x if x.is_contiguous() else x.contiguous()
+    if out is None:
+        vals = torch.empty(k, dtype=x.dtype, device=x.device)
+        idx = torch.empty(k, dtype=torch.int64, device=x.device)
+        pay = torch.empty(k, dtype=torch.uint32, device=x.device) if payload is not None else None
+    else:
+        vals, idx, pay = out
+    if payload is not None:
+        if payload.dtype != torch.uint32 or payload.shape[0] != n or not payload.is_cuda:
+            raise ValueError("payload must be a CUDA uint32 tensor of the same length")
+        payload = payload.contiguous()
+    need = int(lib.topk_workspace_bytes(dt, n, k))
+    if need == 0:
+        raise _lib.TopkError(f"invalid arguments for topk (n={n}, k={k})")
+    ws = workspace if workspace is not None else _workspace(x.device, need)
+    st = lib.topk_select(dt, _ptr(x), _ptr(payload), n, base, k,
+                         _lib.LARGEST if largest else _lib.SMALLEST,
+                         _lib.MODE_FILTER if mode == "filter" else _lib.MODE_PURE,
+                         _ptr(vals), _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
+                         _stream_ptr(x.device))
+    _lib.check(st, "topk_select")
+    return (vals, idx) if payload is None else (vals, idx, pay)
+
+
+def merge(cand_keys: torch.Tensor, cand_idx: torch.Tensor, k: int, largest: bool = True,
+          cand_payload: torch.Tensor | None = None, runs: int = 1):
+    """Exact top-k of candidate entries (key, global int64 index[, payload]) -- the
+    global step after per-partition top-k (multi-GPU all-gather result)."""
+    lib = _lib.load()
+    dt = _dtype_code(cand_keys)
+    total = cand_keys.shape[0]
+    if total % runs:
+        raise ValueError("candidates must be runs * run_len long")
+    cand_keys = cand_keys.contiguous()
+    cand_idx = cand_idx.to(torch.int64).contiguous()
+    dev = cand_keys.device
+    vals = torch.empty(k, dtype=cand_keys.dtype, device=dev)
+    idx = torch.empty(k, dtype=torch.int64, device=dev)
+    pay = None
+    if cand_payload is not None:
+        cand_payload = cand_payload.contiguous()
+        pay = torch.empty(k, dtype=torch.uint32, device=dev)
+    st = lib.topk_merge(dt, _ptr(cand_keys), _ptr(cand_idx), _ptr(cand_payload), runs,
+                        total // runs, k, _lib.LARGEST if largest else _lib.SMALLEST,
+                        _ptr(vals), _ptr(pay), _ptr(idx), None, 0, _stream_ptr(dev))
+    _lib.check(st, "topk_merge")
+    return (vals, idx) if cand_payload is None else (vals, idx, pay)
+
+
+def launch_count() -> int:
+    """Kernels launched by libtopk_b200.so so far in this process."""
+    return int(_lib.load().topk_launch_count())

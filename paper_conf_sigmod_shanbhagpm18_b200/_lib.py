@@ -1,0 +1,76 @@
+"""ctypes binding of include/topk.h (argument marshalling only).
+
+Every step of the top-k runs in libtopk_b200.so's sm_100a kernels; torch provides the
+device memory and the current CUDA stream.  There is no CPU fallback: if the library
+cannot be loaded the call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from . import _build
+
+TOPK_OK = 0
+STATUS = {0: "TOPK_OK", 1: "TOPK_ERR_INVALID_ARG", 2: "TOPK_ERR_UNSUPPORTED",
+          3: "TOPK_ERR_WORKSPACE", 4: "TOPK_ERR_CUDA"}
+F32, U32, F64 = 0, 1, 2
+LARGEST, SMALLEST = 0, 1
+MODE_FILTER, MODE_PURE = 0, 1
+
+# Every symbol include/topk.h declares (tests check the .so exports all of them).
+SYMBOLS = (
+    "topk_workspace_bytes", "topk_workspace_init", "topk_select", "topk_f32", "topk_u32",
+    "topk_f64", "topk_u32_kv", "topk_f64_kv", "topk_merge_workspace_bytes", "topk_merge",
+    "topk_launch_count", "topk_status_string", "topk_abi_version",
+)
+
+_lib = None
+
+
+class TopkError(RuntimeError):
+    pass
+
+
+def load(build_if_missing: bool = True):
+    """Load libtopk_b200.so (building it in-tree first if missing or stale)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if build_if_missing:
+        _build.build()
+    if not os.path.exists(_build.LIB):
+        raise TopkError(f"CUDA library missing: {_build.LIB} (run __graft_entry__.build())")
+    lib = ctypes.CDLL(_build.LIB)
+    vp, u64, u32, i32, sz = (ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int,
+                             ctypes.c_size_t)
+    lib.topk_workspace_bytes.argtypes = [i32, u64, u32]
+    lib.topk_workspace_bytes.restype = sz
+    lib.topk_workspace_init.argtypes = [vp, sz, vp]
+    lib.topk_workspace_init.restype = i32
+    lib.topk_select.argtypes = [i32, vp, vp, u64, u64, u32, i32, i32, vp, vp, vp, vp, sz, vp]
+    lib.topk_select.restype = i32
+    for name in ("topk_f32", "topk_u32", "topk_f64"):
+        getattr(lib, name).argtypes = [vp, u64, u32, i32, vp, vp, vp, sz, vp]
+        getattr(lib, name).restype = i32
+    for name in ("topk_u32_kv", "topk_f64_kv"):
+        getattr(lib, name).argtypes = [vp, vp, u64, u32, i32, vp, vp, vp, vp, sz, vp]
+        getattr(lib, name).restype = i32
+    lib.topk_merge_workspace_bytes.argtypes = [i32, u32, u32, u32]
+    lib.topk_merge_workspace_bytes.restype = sz
+    lib.topk_merge.argtypes = [i32, vp, vp, vp, u32, u32, u32, i32, vp, vp, vp, vp, sz, vp]
+    lib.topk_merge.restype = i32
+    lib.topk_launch_count.argtypes = []
+    lib.topk_launch_count.restype = u64
+    lib.topk_status_string.argtypes = [i32]
+    lib.topk_status_string.restype = ctypes.c_char_p
+    lib.topk_abi_version.argtypes = []
+    lib.topk_abi_version.restype = i32
+    _lib = lib
+    return lib
+
+
+def check(status: int, what: str):
+    if status != TOPK_OK:
+        msg = load().topk_status_string(status).decode()
+        raise TopkError(f"{what}: {msg}")

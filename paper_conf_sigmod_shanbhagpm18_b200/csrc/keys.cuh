@@ -1,0 +1,177 @@
+// keys.cuh -- order codes, (code, index) entries and the fast streaming predicate.
+//
+// The paper describes the method "for tuples consisting only of a key" and compares
+// with `x0 < x1` (Alg. 4 line 9).  To make every compare-exchange a total order
+// (bit-exact indices under ties, defined NaN / +-0; R1-R3) the networks
+// compare ENTRIES: (order code, source index), better = larger code, then lower index.
+//
+//  * E32 -- 32-bit codes (f32, u32): one uint64 = code << 32 | ~lidx, so "better" is a
+//    single unsigned 64-bit compare.  lidx is the row offset inside the launch
+//    (< 2^32 - 1); ~lidx makes lower indices larger.  Sentinel (padding, "padded
+//    with min/max value so that they never show up") = 0: code 0 with lidx 0xFFFFFFFF,
+//    worse than every real key, including a real key of code 0.
+//  * E64 -- 64-bit codes (f64): {code, ~lidx}; sentinel = {0, 0}.
+#pragma once
+#include <cstdint>
+
+namespace topk {
+
+struct E32 {
+    uint64_t v;
+    __device__ __forceinline__ static E32 make(uint32_t code, uint32_t lidx) {
+        return E32{(static_cast<uint64_t>(code) << 32) | static_cast<uint32_t>(~lidx)};
+    }
+    __device__ __forceinline__ static E32 sentinel() { return E32{0ull}; }
+    __device__ __forceinline__ bool is_sentinel() const { return v == 0ull; }
+    __device__ __forceinline__ uint32_t lidx() const { return ~static_cast<uint32_t>(v); }
+    __device__ __forceinline__ uint64_t code() const { return v >> 32; }
+};
+__device__ __forceinline__ bool better(E32 a, E32 b) { return a.v > b.v; }
+
+struct E64 {
+    uint64_t c;
+    uint32_t ni;
+    __device__ __forceinline__ static E64 make(uint64_t code, uint32_t lidx) {
+        return E64{code, ~lidx};
+    }
+    __device__ __forceinline__ static E64 sentinel() { return E64{0ull, 0u}; }
+    __device__ __forceinline__ bool is_sentinel() const { return c == 0ull && ni == 0u; }
+    __device__ __forceinline__ uint32_t lidx() const { return ~ni; }
+    __device__ __forceinline__ uint64_t code() const { return c; }
+};
+__device__ __forceinline__ bool better(E64 a, E64 b) {
+    return a.c > b.c || (a.c == b.c && a.ni > b.ni);
+}
+
+// Shared-memory arrays of entries (structure of arrays for E64: 12 B per entry).
+template <class E>
+struct SBuf;
+template <>
+struct SBuf<E32> {
+    uint64_t* v;
+    static constexpr int kBytes = 8;
+    __device__ __forceinline__ void init(unsigned char* base, int cap) {
+        v = reinterpret_cast<uint64_t*>(base);
+        (void)cap;
+    }
+    __device__ __forceinline__ E32 ld(int i) const { return E32{v[i]}; }
+    __device__ __forceinline__ void st(int i, E32 e) const { v[i] = e.v; }
+};
+template <>
+struct SBuf<E64> {
+    uint64_t* c;
+    uint32_t* ni;
+    static constexpr int kBytes = 12;
+    __device__ __forceinline__ void init(unsigned char* base, int cap) {
+        c = reinterpret_cast<uint64_t*>(base);
+        ni = reinterpret_cast<uint32_t*>(base + 8 * static_cast<size_t>(cap));
+    }
+    __device__ __forceinline__ E64 ld(int i) const { return E64{c[i], ni[i]}; }
+    __device__ __forceinline__ void st(int i, E64 e) const {
+        c[i] = e.c;
+        ni[i] = e.ni;
+    }
+};
+
+// ---------------------------------------------------------------------------------
+// Key traits: code(), threshold decode and the streaming fast test.
+//
+// code_max(x): order-preserving unsigned image (R2).  IEEE-754 patterns of
+// non-negative numbers grow with the value -> set the top bit; negative patterns
+// shrink -> complement.  Overrides: every NaN -> all ones (ranks above +inf, all NaNs
+// tie); -0 -> the code of +0.  Min order uses ~code_max(x).
+//
+// fast<MIN, STRICT>(x, t): a superset test "x may beat the threshold key t", used on
+// every streamed key (1 FSETP/ISETP per key).  For floats the unordered variants
+// (GTU/GEU/LTU/LEU) keep NaN keys, which the exact entry test then decides.
+// ---------------------------------------------------------------------------------
+template <class K>
+struct KeyTraits;
+
+template <>
+struct KeyTraits<float> {
+    using Key = float;
+    using E = E32;
+    using Vec = float4;
+    static constexpr int kVec = 4;
+    __device__ __forceinline__ static uint32_t code_max(float x) {
+        uint32_t u = __float_as_uint(x);
+        uint32_t c = (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+        if (x == 0.0f) c = 0x80000000u;
+        if (x != x) c = 0xFFFFFFFFu;
+        return c;
+    }
+    template <bool MIN>
+    __device__ __forceinline__ static uint32_t code(float x) {
+        return MIN ? ~code_max(x) : code_max(x);
+    }
+    // A key whose code equals `c` (NaN if c is the NaN code).
+    template <bool MIN>
+    __device__ __forceinline__ static float decode(uint64_t c64) {
+        uint32_t c = static_cast<uint32_t>(c64);
+        if (MIN) c = ~c;
+        if (c == 0xFFFFFFFFu) return __uint_as_float(0x7FC00000u);
+        uint32_t u = (c & 0x80000000u) ? (c & 0x7FFFFFFFu) : ~c;
+        return __uint_as_float(u);
+    }
+    template <bool MIN, bool STRICT>
+    __device__ __forceinline__ static bool fast(float x, float t) {
+        if (MIN) return STRICT ? !(x >= t) : !(x > t);
+        return STRICT ? !(x <= t) : !(x < t);
+    }
+};
+
+template <>
+struct KeyTraits<uint32_t> {
+    using Key = uint32_t;
+    using E = E32;
+    using Vec = uint4;
+    static constexpr int kVec = 4;
+    template <bool MIN>
+    __device__ __forceinline__ static uint32_t code(uint32_t x) {
+        return MIN ? ~x : x;
+    }
+    template <bool MIN>
+    __device__ __forceinline__ static uint32_t decode(uint64_t c64) {
+        uint32_t c = static_cast<uint32_t>(c64);
+        return MIN ? ~c : c;
+    }
+    template <bool MIN, bool STRICT>
+    __device__ __forceinline__ static bool fast(uint32_t x, uint32_t t) {
+        if (MIN) return STRICT ? (x < t) : (x <= t);
+        return STRICT ? (x > t) : (x >= t);
+    }
+};
+
+template <>
+struct KeyTraits<double> {
+    using Key = double;
+    using E = E64;
+    using Vec = double2;
+    static constexpr int kVec = 2;
+    __device__ __forceinline__ static uint64_t code_max(double x) {
+        uint64_t u = static_cast<uint64_t>(__double_as_longlong(x));
+        uint64_t c = (u >> 63) ? ~u : (u | 0x8000000000000000ull);
+        if (x == 0.0) c = 0x8000000000000000ull;
+        if (x != x) c = ~0ull;
+        return c;
+    }
+    template <bool MIN>
+    __device__ __forceinline__ static uint64_t code(double x) {
+        return MIN ? ~code_max(x) : code_max(x);
+    }
+    template <bool MIN>
+    __device__ __forceinline__ static double decode(uint64_t c) {
+        if (MIN) c = ~c;
+        if (c == ~0ull) return __longlong_as_double(0x7FF8000000000000ll);
+        uint64_t u = (c >> 63) ? (c & 0x7FFFFFFFFFFFFFFFull) : ~c;
+        return __longlong_as_double(static_cast<long long>(u));
+    }
+    template <bool MIN, bool STRICT>
+    __device__ __forceinline__ static bool fast(double x, double t) {
+        if (MIN) return STRICT ? !(x >= t) : !(x > t);
+        return STRICT ? !(x <= t) : !(x < t);
+    }
+};
+
+}  // namespace topk

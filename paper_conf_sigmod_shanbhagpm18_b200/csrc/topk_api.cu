@@ -1,0 +1,286 @@
+// topk_api.cu -- the C ABI declared in include/topk.h: argument validation, planning
+// (alignment peel, tiles, grid, tile permutation), workspace layout, and dispatch of
+// the sm_100a kernels.  No host synchronisation, no allocation.
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+#include <cstring>
+
+#include "merge.cuh"
+#include "select.cuh"
+#include "topk.h"
+
+namespace {
+
+std::atomic<uint64_t> g_launches{0};
+
+struct DevInfo {
+    int sms = 0;
+    int major = 0;
+    bool ok = false;
+};
+DevInfo g_dev[64];
+
+bool device_info(int* sms, int* major) {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return false;
+    DevInfo& d = g_dev[dev];
+    if (!d.ok) {
+        if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+            return false;
+        if (cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, dev) !=
+            cudaSuccess)
+            return false;
+        d.ok = true;
+    }
+    *sms = d.sms;
+    *major = d.major;
+    return true;
+}
+
+size_t key_size(topk_dtype_t dt) { return dt == TOPK_F64 ? 8 : 4; }
+size_t entry_bytes(topk_dtype_t dt) { return dt == TOPK_F64 ? 12 : 8; }
+
+uint32_t next_pow2_u32(uint32_t x) {
+    uint32_t p = 1;
+    while (p < x) p <<= 1;
+    return p;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+bool valid_dtype(int dt) { return dt == TOPK_F32 || dt == TOPK_U32 || dt == TOPK_F64; }
+bool valid_order(int o) { return o == TOPK_LARGEST || o == TOPK_SMALLEST; }
+
+// Largest n one launch indexes with a 32-bit local row id (0xFFFFFFFF is reserved for
+// the sentinel entry).
+constexpr uint64_t kMaxLaunchN = 0xFFFFFFFEull;
+
+template <class Key, bool MIN, bool FILTER>
+cudaError_t launch_select(const topk::SelectParams& p, int grid, cudaStream_t st) {
+    static bool attr_set = false;  // per instantiation (benign race: idempotent)
+    const size_t smem = topk::select_smem_bytes<Key>();
+    if (!attr_set) {
+        cudaError_t e = cudaFuncSetAttribute(topk::select_kernel<Key, MIN, FILTER>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             static_cast<int>(smem));
+        if (e != cudaSuccess) return e;
+        attr_set = true;
+    }
+    topk::select_kernel<Key, MIN, FILTER><<<grid, topk::kNT, smem, st>>>(p);
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return cudaGetLastError();
+}
+
+template <class Key>
+cudaError_t dispatch_select(const topk::SelectParams& p, int grid, bool min_order, bool filter,
+                            cudaStream_t st) {
+    if (min_order)
+        return filter ? launch_select<Key, true, true>(p, grid, st)
+                      : launch_select<Key, true, false>(p, grid, st);
+    return filter ? launch_select<Key, false, true>(p, grid, st)
+                  : launch_select<Key, false, false>(p, grid, st);
+}
+
+template <class Key, bool MIN>
+cudaError_t launch_merge(const topk::MergeParams& p, cudaStream_t st) {
+    static bool attr_set = false;
+    if (!attr_set) {
+        cudaError_t e = cudaFuncSetAttribute(topk::merge_kernel<Key, MIN>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             static_cast<int>(topk::kMergeSmem));
+        if (e != cudaSuccess) return e;
+        attr_set = true;
+    }
+    topk::merge_kernel<Key, MIN><<<1, topk::kMergeNT, topk::kMergeSmem, st>>>(p);
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return cudaGetLastError();
+}
+
+template <class Key>
+cudaError_t dispatch_merge(const topk::MergeParams& p, bool min_order, cudaStream_t st) {
+    return min_order ? launch_merge<Key, true>(p, st) : launch_merge<Key, false>(p, st);
+}
+
+template <class Key>
+uint32_t tile_keys() {
+    return static_cast<uint32_t>(topk::Cfg<Key>::kTileKeys);
+}
+
+uint32_t tile_keys_for(topk_dtype_t dt) {
+    switch (dt) {
+        case TOPK_F64: return tile_keys<double>();
+        case TOPK_U32: return tile_keys<uint32_t>();
+        default: return tile_keys<float>();
+    }
+}
+
+}  // namespace
+
+extern "C" {
+
+size_t topk_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k) {
+    if (!valid_dtype(dtype) || n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return 0;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return 0;
+    return align_up(sizeof(topk::WsHeader) + static_cast<size_t>(sms) * k * entry_bytes(dtype),
+                    256);
+}
+
+topk_status_t topk_workspace_init(void* ws, size_t ws_bytes, void* stream) {
+    if (!ws || ws_bytes < sizeof(topk::WsHeader)) return TOPK_ERR_WORKSPACE;
+    if (cudaMemsetAsync(ws, 0, ws_bytes, static_cast<cudaStream_t>(stream)) != cudaSuccess)
+        return TOPK_ERR_CUDA;
+    return TOPK_OK;
+}
+
+topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
+                          uint64_t n, uint64_t base, uint32_t k, topk_order_t order,
+                          topk_mode_t mode, void* out_keys, uint32_t* out_payload,
+                          int64_t* out_idx, void* ws, size_t ws_bytes, void* stream) {
+    if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
+    if (mode != TOPK_MODE_FILTER && mode != TOPK_MODE_PURE) return TOPK_ERR_INVALID_ARG;
+    if (!keys || n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return TOPK_ERR_INVALID_ARG;
+    if (out_payload && !payload) return TOPK_ERR_INVALID_ARG;
+    const size_t ks = key_size(dtype);
+    const uintptr_t addr = reinterpret_cast<uintptr_t>(keys);
+    if (addr % ks) return TOPK_ERR_INVALID_ARG;
+    if (n > kMaxLaunchN) return TOPK_ERR_UNSUPPORTED;  // chunked path: see DESIGN.md §9
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    if (major != 10) return TOPK_ERR_UNSUPPORTED;
+    const size_t need = topk_workspace_bytes(dtype, n, k);
+    if (!ws || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws) % 256)) return TOPK_ERR_WORKSPACE;
+
+    topk::SelectParams p;
+    std::memset(&p, 0, sizeof(p));
+    p.keys = keys;
+    p.payload = payload;
+    p.out_keys = out_keys;
+    p.out_payload = out_payload;
+    p.out_idx = out_idx;
+    p.ws = static_cast<unsigned char*>(ws);
+    p.n = n;
+    p.base = base;
+    const uint64_t vec = 16 / ks;
+    uint64_t head = ((16 - (addr % 16)) % 16) / ks;
+    if (head > n) head = n;
+    p.head = static_cast<uint32_t>(head);
+    p.body_n = (n - head) / vec * vec;
+    const uint32_t tk = tile_keys_for(dtype);
+    const uint64_t ntiles = (p.body_n + tk - 1) / tk;
+    p.ntiles = static_cast<uint32_t>(ntiles);
+    p.k = k;
+    p.K = next_pow2_u32(k);
+    // Tile permutation half-width: 2h bits cover ntiles.
+    uint32_t bits = 0;
+    while ((1ull << bits) < ntiles) ++bits;
+    p.perm_h = ntiles > 1 ? (bits + 1) / 2 : 0;
+    const int grid = static_cast<int>(ntiles == 0 ? 1 : (ntiles < (uint64_t)sms ? ntiles : sms));
+
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
+    cudaError_t e;
+    switch (dtype) {
+        case TOPK_F32: e = dispatch_select<float>(p, grid, mn, filt, st); break;
+        case TOPK_U32: e = dispatch_select<uint32_t>(p, grid, mn, filt, st); break;
+        default: e = dispatch_select<double>(p, grid, mn, filt, st); break;
+    }
+    return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+}
+
+topk_status_t topk_f32(const float* keys, uint64_t n, uint32_t k, topk_order_t order,
+                       float* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream) {
+    return topk_select(TOPK_F32, keys, nullptr, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                       nullptr, out_idx, ws, ws_bytes, stream);
+}
+topk_status_t topk_u32(const uint32_t* keys, uint64_t n, uint32_t k, topk_order_t order,
+                       uint32_t* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream) {
+    return topk_select(TOPK_U32, keys, nullptr, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                       nullptr, out_idx, ws, ws_bytes, stream);
+}
+topk_status_t topk_f64(const double* keys, uint64_t n, uint32_t k, topk_order_t order,
+                       double* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream) {
+    return topk_select(TOPK_F64, keys, nullptr, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                       nullptr, out_idx, ws, ws_bytes, stream);
+}
+topk_status_t topk_u32_kv(const uint32_t* keys, const uint32_t* payload, uint64_t n,
+                          uint32_t k, topk_order_t order, uint32_t* out_keys,
+                          uint32_t* out_payload, int64_t* out_idx, void* ws,
+                          size_t ws_bytes, void* stream) {
+    return topk_select(TOPK_U32, keys, payload, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                       out_payload, out_idx, ws, ws_bytes, stream);
+}
+topk_status_t topk_f64_kv(const double* keys, const uint32_t* payload, uint64_t n,
+                          uint32_t k, topk_order_t order, double* out_keys,
+                          uint32_t* out_payload, int64_t* out_idx, void* ws,
+                          size_t ws_bytes, void* stream) {
+    return topk_select(TOPK_F64, keys, payload, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                       out_payload, out_idx, ws, ws_bytes, stream);
+}
+
+size_t topk_merge_workspace_bytes(topk_dtype_t dtype, uint32_t runs, uint32_t run_len,
+                                  uint32_t k) {
+    (void)dtype;
+    (void)runs;
+    (void)run_len;
+    (void)k;
+    return 256;  // the merge runs in one CTA's shared memory; reserved for future use
+}
+
+topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_t* cand_idx,
+                         const uint32_t* cand_payload, uint32_t runs, uint32_t run_len,
+                         uint32_t k, topk_order_t order, void* out_keys,
+                         uint32_t* out_payload, int64_t* out_idx, void* ws,
+                         size_t ws_bytes, void* stream) {
+    (void)ws;
+    (void)ws_bytes;
+    if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
+    if (!cand_keys || !cand_idx || runs == 0 || run_len == 0) return TOPK_ERR_INVALID_ARG;
+    const uint64_t total = static_cast<uint64_t>(runs) * run_len;
+    if (total > 65536 || k == 0 || k > TOPK_MAX_K || k > total) return TOPK_ERR_INVALID_ARG;
+    if (out_payload && !cand_payload) return TOPK_ERR_INVALID_ARG;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    if (major != 10) return TOPK_ERR_UNSUPPORTED;
+    topk::MergeParams p;
+    p.cand_keys = cand_keys;
+    p.cand_idx = cand_idx;
+    p.cand_payload = cand_payload;
+    p.out_keys = out_keys;
+    p.out_payload = out_payload;
+    p.out_idx = out_idx;
+    p.total = static_cast<uint32_t>(total);
+    p.k = k;
+    p.K = next_pow2_u32(k);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const bool mn = order == TOPK_SMALLEST;
+    cudaError_t e;
+    switch (dtype) {
+        case TOPK_F32: e = dispatch_merge<float>(p, mn, st); break;
+        case TOPK_U32: e = dispatch_merge<uint32_t>(p, mn, st); break;
+        default: e = dispatch_merge<double>(p, mn, st); break;
+    }
+    return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+}
+
+uint64_t topk_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
+
+const char* topk_status_string(topk_status_t s) {
+    switch (s) {
+        case TOPK_OK: return "TOPK_OK";
+        case TOPK_ERR_INVALID_ARG: return "TOPK_ERR_INVALID_ARG: invalid argument";
+        case TOPK_ERR_UNSUPPORTED: return "TOPK_ERR_UNSUPPORTED: device or size not supported";
+        case TOPK_ERR_WORKSPACE: return "TOPK_ERR_WORKSPACE: workspace NULL, too small or misaligned";
+        case TOPK_ERR_CUDA: return "TOPK_ERR_CUDA: CUDA runtime or launch error";
+    }
+    return "unknown topk_status_t";
+}
+
+int topk_abi_version(void) { return TOPK_ABI_VERSION; }
+
+}  // extern "C"
