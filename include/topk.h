@@ -128,6 +128,14 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
                          uint32_t* out_payload, int64_t* out_idx, void* ws,
                          size_t ws_bytes, void* stream);
 
+/* Read-bandwidth probe (the paper's "Memory Bandwidth" line: the time to read
+ * the data once, a lower bound for any top-k): reads `bytes` (multiple of 16, 16-byte
+ * aligned) at `data` once.  method 0: 128-bit non-coherent loads, `grid` CTAs of 512
+ * threads (0 = 4 per SM); method 1: the top-k pass's TMA ring (`tile` bytes x `stages`,
+ * one CTA per SM).  `sink` is a device uint32 (scratch).  Enqueued on `stream`. */
+topk_status_t topk_probe_read(const void* data, size_t bytes, int method, int grid, int tile,
+                              int stages, uint32_t* sink, void* stream);
+
 /* Number of kernels this library has launched in this process (for the bench's
  * "gpu_launches" count).  Thread-safe, monotone. */
 uint64_t topk_launch_count(void);

@@ -22,7 +22,7 @@ MODE_FILTER, MODE_PURE = 0, 1
 SYMBOLS = (
     "topk_workspace_bytes", "topk_workspace_init", "topk_select", "topk_f32", "topk_u32",
     "topk_f64", "topk_u32_kv", "topk_f64_kv", "topk_merge_workspace_bytes", "topk_merge",
-    "topk_launch_count", "topk_status_string", "topk_abi_version",
+    "topk_launch_count", "topk_status_string", "topk_abi_version", "topk_probe_read",
 )
 
 _lib = None
@@ -37,11 +37,14 @@ def load(build_if_missing: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    if build_if_missing:
-        _build.build()
-    if not os.path.exists(_build.LIB):
-        raise TopkError(f"CUDA library missing: {_build.LIB} (run __graft_entry__.build())")
-    lib = ctypes.CDLL(_build.LIB)
+    path = os.environ.get("TOPK_LIB")  # dev: load an alternative in-tree build
+    if path is None:
+        if build_if_missing:
+            _build.build()
+        path = _build.LIB
+    if not os.path.exists(path):
+        raise TopkError(f"CUDA library missing: {path} (run __graft_entry__.build())")
+    lib = ctypes.CDLL(path)
     vp, u64, u32, i32, sz = (ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int,
                              ctypes.c_size_t)
     lib.topk_workspace_bytes.argtypes = [i32, u64, u32]
@@ -60,6 +63,8 @@ def load(build_if_missing: bool = True):
     lib.topk_merge_workspace_bytes.restype = sz
     lib.topk_merge.argtypes = [i32, vp, vp, vp, u32, u32, u32, i32, vp, vp, vp, vp, sz, vp]
     lib.topk_merge.restype = i32
+    lib.topk_probe_read.argtypes = [vp, sz, i32, i32, i32, i32, vp, vp]
+    lib.topk_probe_read.restype = i32
     lib.topk_launch_count.argtypes = []
     lib.topk_launch_count.restype = u64
     lib.topk_status_string.argtypes = [i32]

@@ -43,7 +43,35 @@ __device__ __forceinline__ bool better(E64 a, E64 b) {
     return a.c > b.c || (a.c == b.c && a.ni > b.ni);
 }
 
+// Branch-free select (selp): the compiler otherwise turns data-dependent swaps into
+// divergent branches, serialising the warp.
+__device__ __forceinline__ uint64_t sel64(bool p, uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\tselp.b64 %0, %1, %2, q;\n\t}"
+        : "=l"(r)
+        : "l"(a), "l"(b), "r"(static_cast<uint32_t>(p)));
+    return r;
+}
+__device__ __forceinline__ uint32_t sel32(bool p, uint32_t a, uint32_t b) {
+    uint32_t r;
+    asm("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %3, 0;\n\tselp.b32 %0, %1, %2, q;\n\t}"
+        : "=r"(r)
+        : "r"(a), "r"(b), "r"(static_cast<uint32_t>(p)));
+    return r;
+}
+__device__ __forceinline__ E32 esel(bool p, E32 a, E32 b) { return E32{sel64(p, a.v, b.v)}; }
+__device__ __forceinline__ E64 esel(bool p, E64 a, E64 b) {
+    return E64{sel64(p, a.c, b.c), sel32(p, a.ni, b.ni)};
+}
+
 // Shared-memory arrays of entries (structure of arrays for E64: 12 B per entry).
+// Entry index e is stored at swz(e) = e ^ (((e >> 4) & 7) << 1): the 16-byte column of
+// a 128-byte row is XORed with the row number, so a warp whose lanes each read one
+// 16-entry row (the register networks' blocked layout) hits 8 distinct columns per
+// quarter-warp -- conflict-free (the B200 analogue of the paper's padding / chunk
+// permutation).  Pairs (2j, 2j+1) stay adjacent (16-byte loads).
+__device__ __forceinline__ int swz(int e) { return e ^ (((e >> 4) & 7) << 1); }
+
 template <class E>
 struct SBuf;
 template <>
@@ -54,8 +82,17 @@ struct SBuf<E32> {
         v = reinterpret_cast<uint64_t*>(base);
         (void)cap;
     }
-    __device__ __forceinline__ E32 ld(int i) const { return E32{v[i]}; }
-    __device__ __forceinline__ void st(int i, E32 e) const { v[i] = e.v; }
+    __device__ __forceinline__ E32 ld(int i) const { return E32{v[swz(i)]}; }
+    __device__ __forceinline__ void st(int i, E32 e) const { v[swz(i)] = e.v; }
+    // entries i, i+1 (i even) with one 16-byte access
+    __device__ __forceinline__ void ld2(int i, E32& a, E32& b) const {
+        const ulonglong2 q = *reinterpret_cast<const ulonglong2*>(v + swz(i));
+        a = E32{q.x};
+        b = E32{q.y};
+    }
+    __device__ __forceinline__ void st2(int i, E32 a, E32 b) const {
+        *reinterpret_cast<ulonglong2*>(v + swz(i)) = make_ulonglong2(a.v, b.v);
+    }
 };
 template <>
 struct SBuf<E64> {
@@ -66,10 +103,26 @@ struct SBuf<E64> {
         c = reinterpret_cast<uint64_t*>(base);
         ni = reinterpret_cast<uint32_t*>(base + 8 * static_cast<size_t>(cap));
     }
-    __device__ __forceinline__ E64 ld(int i) const { return E64{c[i], ni[i]}; }
+    __device__ __forceinline__ E64 ld(int i) const {
+        const int j = swz(i);
+        return E64{c[j], ni[j]};
+    }
     __device__ __forceinline__ void st(int i, E64 e) const {
-        c[i] = e.c;
-        ni[i] = e.ni;
+        const int j = swz(i);
+        c[j] = e.c;
+        ni[j] = e.ni;
+    }
+    __device__ __forceinline__ void ld2(int i, E64& a, E64& b) const {
+        const int j = swz(i);
+        const ulonglong2 q = *reinterpret_cast<const ulonglong2*>(c + j);
+        const uint2 n = *reinterpret_cast<const uint2*>(ni + j);
+        a = E64{q.x, n.x};
+        b = E64{q.y, n.y};
+    }
+    __device__ __forceinline__ void st2(int i, E64 a, E64 b) const {
+        const int j = swz(i);
+        *reinterpret_cast<ulonglong2*>(c + j) = make_ulonglong2(a.c, b.c);
+        *reinterpret_cast<uint2*>(ni + j) = make_uint2(a.ni, b.ni);
     }
 };
 

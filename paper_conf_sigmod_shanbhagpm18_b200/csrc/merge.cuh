@@ -20,6 +20,9 @@ struct EM {
 __device__ __forceinline__ bool better(EM a, EM b) {
     return a.c > b.c || (a.c == b.c && a.idx < b.idx);
 }
+__device__ __forceinline__ EM esel(bool p, EM a, EM b) {
+    return EM{sel64(p, a.c, b.c), sel64(p, a.idx, b.idx), sel32(p, a.row, b.row)};
+}
 template <>
 struct SBuf<EM> {
     uint64_t* c;

@@ -1,0 +1,64 @@
+// netbench.cuh -- microbenchmark of the flush networks (dev instrumentation): one CTA
+// of select_kernel's consumer shape sorts P pseudo-random entries to a top-K run,
+// `iters` times, and reports the cycles per network call.
+#pragma once
+#include "network.cuh"
+#include "wnet.cuh"
+
+namespace topk {
+
+template <class E>
+__device__ __forceinline__ E bench_entry(uint32_t i, uint32_t it);
+template <>
+__device__ __forceinline__ E32 bench_entry<E32>(uint32_t i, uint32_t it) {
+    uint32_t h = (i + 1u) * 0x9E3779B1u ^ (it * 0x85EBCA6Bu);
+    h ^= h >> 15;
+    h *= 0x2C1B3C6Du;
+    h ^= h >> 12;
+    return E32::make(h, i);
+}
+template <>
+__device__ __forceinline__ E64 bench_entry<E64>(uint32_t i, uint32_t it) {
+    uint32_t h = (i + 1u) * 0x9E3779B1u ^ (it * 0x85EBCA6Bu);
+    h ^= h >> 15;
+    h *= 0x2C1B3C6Du;
+    h ^= h >> 12;
+    return E64::make((static_cast<uint64_t>(h) << 32) | h, i);
+}
+
+template <class E, int NW>
+__global__ void __launch_bounds__(NW * 32, 1) netbench_kernel(int P, int L, int iters, int smem_net,
+                                                              unsigned long long* out) {
+    extern __shared__ __align__(128) unsigned char smem[];
+    SBuf<E> b;
+    b.init(smem, 4096);
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned long long total = 0;
+    for (int it = 0; it < iters; ++it) {
+        for (int i = threadIdx.x; i < P; i += NW * 32) b.st(i, bench_entry<E>(i, it));
+        NamedSync<NW * 32>::sync();
+        const long long t0 = clock64();
+        if (smem_net == 2) {  // barrier cost: 64 named barriers
+            for (int q = 0; q < 64; ++q) NamedSync<NW * 32>::sync();
+        } else if (smem_net == 3) {  // barrier + one 16-B shared load/store per thread
+            for (int q = 0; q < 64; ++q) {
+                E x0, x1;
+                b.ld2((threadIdx.x * 2 + q * 2) & (P - 1) & ~1, x0, x1);
+                NamedSync<NW * 32>::sync();
+                b.st2((threadIdx.x * 2 + q * 4) & (P - 1) & ~1, x1, x0);
+                NamedSync<NW * 32>::sync();
+            }
+        } else if (smem_net)
+            bitonic_topk_smem<E, NW * 32, NamedSync<NW * 32>>(b, P, 1 << L);
+        else
+            wnet_topk<E, NW, NamedSync<NW * 32>>(b, P, L, w, lane);
+        NamedSync<NW * 32>::sync();
+        total += static_cast<unsigned long long>(clock64() - t0);
+    }
+    if (threadIdx.x == 0) {
+        out[0] = total / iters;
+        out[1] = b.ld(0).code();
+    }
+}
+
+}  // namespace topk

@@ -41,12 +41,10 @@ __device__ __forceinline__ void net_step(const SBuf<E>& b, int P, int inc, int d
         int i = (t << 1) - low;
         int j = i + inc;
         bool best_first = (i & dir) == 0;
-        E x0 = b.ld(i), x1 = b.ld(j);
-        bool sw = best_first ? better(x1, x0) : better(x0, x1);
-        if (sw) {
-            b.st(i, x1);
-            b.st(j, x0);
-        }
+        const E x0 = b.ld(i), x1 = b.ld(j);
+        const bool sw = best_first == better(x1, x0);
+        b.st(i, esel(sw, x1, x0));
+        b.st(j, esel(sw, x0, x1));
     }
     Sync::sync();
 }
@@ -70,7 +68,7 @@ __device__ void bitonic_topk_smem(const SBuf<E>& b, int P, int K) {
             if (t < half) {
                 int i = (t << 1) - (t & (K - 1));  // element p of run 2q, partner in run 2q+1
                 E a = b.ld(i), c = b.ld(i + K);
-                keep[r] = better(a, c) ? a : c;
+                keep[r] = esel(better(a, c), a, c);
             }
         }
         Sync::sync();

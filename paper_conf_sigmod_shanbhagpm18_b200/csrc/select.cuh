@@ -1,43 +1,66 @@
-// select.cuh -- the fused streaming pass: one persistent CTA per SM reads its share of
-// the input from HBM exactly once (1-D bulk TMA into a shared-memory ring), keeps the
-// keys that can still be in the top-k, and runs the paper's local sort / merge /
-// rebuild network over the kept keys together with its running top-K run.  The last
-// CTA to finish reduces all CTAs' runs and writes the result (the paper's
-// "SortReducer then BitonicReducer until k remain", P:179-180 / P:327, fused into one
-// launch: the intermediate candidates live in L2, never in a second HBM pass).
+// select.cuh -- the fused streaming pass of bitonic top-k.
 //
-// CTA = 16 consumer warps + 1 producer warp.
-//   * Producer (one lane): for each of the CTA's tiles -- assigned round-robin through
-//     a fixed pseudo-random permutation so that no input order (sorted, reversed) lines
-//     up with the scan (the robustness the paper claims for the pure method, P:264/268,
-//     is kept by the filter path) -- waits for the ring slot to be empty, issues the
-//     bulk copy, and publishes the slot's metadata: tile id and the current threshold
-//     (max of the CTA's own k-th best and the global tau_g).
-//   * Consumers: per key one compare against the threshold key t (fast test, a superset
-//     of "can still be in the top-k"); for the few passing keys the exact entry test
-//     and a warp-aggregated append into the survivor buffer (the paper's "buffer
-//     filler": prefix sum of matches into a shared-memory buffer).  The buffer
-//     is flushed -- bitonic top-K of [running run | survivors | sentinel padding], the
-//     paper's local sort + merge + rebuild (network.cuh) -- when it fills; a warp whose
-//     survivors do not fit keeps its ring slot, and redoes the tile after the flush.
-//   * After each flush the CTA's k-th best is published to tau_g (atomic max): every
-//     CTA's k-th best is a valid lower bound of the global k-th best.
+// One persistent CTA per SM reads its share of the input from HBM exactly once (1-D
+// bulk TMA into a shared-memory ring), keeps the keys that can still be in the top-k,
+// and runs the paper's local sort / merge / rebuild network (wnet.cuh, network.cuh)
+// over the kept keys together with its running top-K run.  The last CTA to finish
+// reduces all CTAs' runs and writes the result.  This is the paper's "SortReducer,
+// then BitonicReducer until k remain" fused into one launch: the
+// intermediate candidates live on chip / in L2, never in a second HBM pass.
+//
+// CTA = 15 consumer warps + 1 producer warp (16 warps: 4 per SM sub-partition, so a
+// thread may use 128 registers).
+//   * Producer warp: claims blocks of tiles from a global counter (fast SMs take more),
+//     visits waves of blocks in a fixed pseudo-random order -- all SMs stream one
+//     address window at a time (DRAM row locality) while no input order (sorted,
+//     reversed) lines up with the scan, keeping the robustness the paper claims for
+//     the pure method -- and issues one bulk copy per ring slot.
+//   * Consumers: per key one compare against the threshold key t (fast test, a
+//     superset of "can still be in the top-k"); for the few passing keys the exact
+//     entry test and a warp-aggregated append into the survivor buffer -- the paper's
+//     "buffer filler": a prefix sum of matches into a shared-memory buffer,
+//     with the predicate "better than the current bound".
+//   * When an append does not fit, the warp requests a collective flush: bitonic
+//     top-K of [running run | survivors | sentinel padding].  No per-tile barrier: the
+//     other warps join at their next wait point (tile wait or final drain); the
+//     requesting warp keeps its ring slot and redoes its share of the tile afterwards.
+//   * The bound: the CTA's own k-th best, every other CTA's k-th best (tau_g), and a
+//     rank bound over every CTA's published run samples (the 2^j-th best of each run):
+//     if t runs have a 2^j-th best >= v, then >= t * 2^j entries are >= v, so the t-th
+//     largest sample of row j, t = ceil(k / 2^j), bounds the global k-th best.  All
+//     bounds are entries owned by some run, so a strict test against them never drops
+//     a top-k entry.
 #pragma once
 #include "keys.cuh"
 #include "network.cuh"
 #include "ptx.cuh"
+#include "wnet.cuh"
 
 namespace topk {
 
-constexpr int kNC = 512;              // consumer threads (16 warps)
-constexpr int kNT = kNC + 32;         // + one producer warp
-constexpr int kTileBytes = 32768;     // bytes per TMA stage
-constexpr int kStages = 4;            // ring depth
-constexpr int kCap = 8192;            // survivor buffer entries (incl. the running run)
+#ifndef TOPK_VEC_PER_THREAD
+#define TOPK_VEC_PER_THREAD 4
+#endif
+#ifndef TOPK_STAGES
+#define TOPK_STAGES 5
+#endif
+#ifndef TOPK_REFRESH_AT
+#define TOPK_REFRESH_AT 12  // tile index at which warp 0 requests a rank-bound refresh
+#endif
+
+constexpr int kNC = 480;                                    // consumer threads (15 warps)
+constexpr int kNT = kNC + 32;                               // + one producer warp
+constexpr int kTileBytes = kNC * 16 * TOPK_VEC_PER_THREAD;  // 30 KB per TMA stage
+constexpr int kStagesMax = TOPK_STAGES;
+constexpr int kCap = 4096;            // survivor buffer entries (incl. the running run)
+constexpr int kPubRows = 11;          // published 2^j-th best for j <= log2(1024)
+constexpr int kGMax = 160;            // CTAs (>= SM count)
+constexpr int kScratch = kPubRows * kGMax;  // shared: staged samples (u64)
 using CSync = NamedSync<kNC>;
 
 template <class Key>
 struct Cfg {
+    static constexpr int kStages = sizeof(Key) == 8 ? TOPK_STAGES - 1 : TOPK_STAGES;
     static constexpr int kTileKeys = kTileBytes / static_cast<int>(sizeof(Key));
     static constexpr int kVecPerThread = kTileBytes / 16 / kNC;
     static constexpr int kItems = kTileKeys / kNC;  // keys per consumer thread per tile
@@ -45,9 +68,10 @@ struct Cfg {
 };
 
 struct WsHeader {
-    unsigned long long tau_g;  // global threshold: max over CTAs of their k-th best
+    unsigned long long tau_g;  // max over CTAs of their k-th best
     unsigned int ticket;       // CTAs finished
-    unsigned int pad[13];
+    unsigned int next_tile;    // dynamic work claiming counter
+    unsigned int pad[12];
 };
 static_assert(sizeof(WsHeader) == 64, "header");
 
@@ -64,9 +88,20 @@ struct SelectParams {
     uint32_t head;     // unaligned leading keys (processed as extras by CTA 0)
     uint32_t ntiles;   // tiles of the body
     uint32_t k, K;     // requested k and K = next_pow2(k)
-    uint32_t perm_h;   // Feistel half-width (bits); 0 = identity tile order
-    uint32_t pad;
+    uint32_t perm_h;   // Feistel half-width (bits) over nwaves; 0 = identity order
+    uint32_t blk;      // tiles per claimed block
+    uint32_t nblocks;  // ceil(ntiles / blk)
+    uint32_t wave;     // blocks per wave (permutation unit)
+    uint32_t nwaves;   // ceil(nblocks / wave)
+    uint32_t gmax;     // workspace layout: published-sample columns (>= gridDim.x)
+    uint32_t J;        // published samples per CTA: the 2^j-th best of its run, j < J
 };
+
+// Workspace: [WsHeader | pub: u64[kPubRows][gmax] | cand: G x k entries]
+__host__ __device__ constexpr size_t ws_pub_offset() { return 64; }
+__host__ __device__ inline size_t ws_cand_offset(uint32_t gmax) {
+    return 64 + static_cast<size_t>(kPubRows) * gmax * 8;
+}
 
 // Global (workspace) candidate storage, structure of arrays like SBuf.
 template <class E>
@@ -96,26 +131,21 @@ struct GBuf<E64> {
     }
 };
 
-// Global threshold publish / read.  E32: the packed entry (exact, with its index).
-// E64: the code only, read back as {code, ni = 0} -- i.e. non-strict on that code.
+// Bounds as 64-bit words: E32 the packed entry (exact, index included); E64 the code
+// only, read back as {code, ni = 0} -- i.e. non-strict on that code (still valid).
+__device__ __forceinline__ unsigned long long bound_word(E32 e) { return e.v; }
+__device__ __forceinline__ unsigned long long bound_word(E64 e) { return e.c; }
+template <class E>
+__device__ __forceinline__ E from_bound_word(unsigned long long w);
+template <>
+__device__ __forceinline__ E32 from_bound_word<E32>(unsigned long long w) { return E32{w}; }
+template <>
+__device__ __forceinline__ E64 from_bound_word<E64>(unsigned long long w) { return E64{w, 0u}; }
 __device__ __forceinline__ void tau_publish(WsHeader* h, E32 e) { atomicMax(&h->tau_g, e.v); }
 __device__ __forceinline__ void tau_publish(WsHeader* h, E64 e) { atomicMax(&h->tau_g, e.c); }
-template <class E>
-__device__ __forceinline__ E tau_from_raw(uint64_t raw);
-template <>
-__device__ __forceinline__ E32 tau_from_raw<E32>(uint64_t raw) { return E32{raw}; }
-template <>
-__device__ __forceinline__ E64 tau_from_raw<E64>(uint64_t raw) { return E64{raw, 0u}; }
-__device__ __forceinline__ uint64_t tau_load_raw(const WsHeader* h) {
-    return ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&h->tau_g));
-}
 
-__device__ __forceinline__ E32 load_volatile(const E32* e) {
-    return E32{*reinterpret_cast<const volatile uint64_t*>(&e->v)};
-}
-__device__ __forceinline__ E64 load_volatile(const E64* e) {
-    return E64{*reinterpret_cast<const volatile uint64_t*>(&e->c),
-               *reinterpret_cast<const volatile uint32_t*>(&e->ni)};
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
 // Threshold parameters derived from a bound tau.
@@ -138,16 +168,8 @@ __device__ __forceinline__ Par<typename KeyTraits<Key>::E, Key> make_par(
     return p;
 }
 
-// Metadata the producer publishes with each ring slot.
-template <class E, class Key>
-struct SlotMeta {
-    Par<E, Key> par;
-    uint32_t tlen;   // keys in this tile
-    uint32_t lbase;  // launch-relative row of the tile's first key
-};
-
-// Bijection on [0, ntiles): 4-round Feistel on 2h bits with cycle walking.
-__device__ __forceinline__ uint32_t tile_of(uint32_t i, uint32_t ntiles, uint32_t h) {
+// Bijection on [0, n): 4-round Feistel on 2h bits with cycle walking.
+__device__ __forceinline__ uint32_t feistel_perm(uint32_t i, uint32_t n, uint32_t h) {
     if (h == 0) return i;
     const uint32_t mask = (1u << h) - 1u;
     uint32_t x = i;
@@ -159,12 +181,12 @@ __device__ __forceinline__ uint32_t tile_of(uint32_t i, uint32_t ntiles, uint32_
             f ^= f >> 15;
             f *= 0x2C1B3C6Du;
             f ^= f >> 12;
-            uint32_t nl = R;
+            const uint32_t nl = R;
             R = L ^ (f & mask);
             L = nl;
         }
         x = (L << h) | R;
-    } while (x >= ntiles);
+    } while (x >= n);
     return x;
 }
 
@@ -199,47 +221,78 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }
 
+constexpr uint32_t kEndTile = 0xFFFFFFFFu;
+constexpr int kReqFlush = 1, kReqRefresh = 2;
+
 // Shared state of one CTA.
 template <class E, class Key>
 struct CtaState {
-    int cnt;          // survivors in buf[K ..)
-    int last;         // this CTA reduces all candidates
-    uint32_t tau_ver; // seqlock over tau (producer reads it without a barrier)
-    E tau;            // CTA bound: its own k-th best, or better
-    SlotMeta<E, Key> meta[kStages];
+    int cnt;                   // survivors in buf[K ..)
+    int req;                   // collective requests (kReqFlush | kReqRefresh)
+    int nflush;                // flushes done
+    int last;                  // this CTA reduces all candidates
+    unsigned long long tau_w;  // E32: the bound as one packed word
+    E tau;                     // E64: the bound
+    Par<E, Key> par;           // E64: fast-test parameters of tau
+    unsigned long long best[kPubRows];
+    uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
 };
 
-// Reserve `total` entries of the survivor buffer (lane 31 of the warp), or fail (-1)
-// if they do not fit; the caller then keeps its slot and retries after a flush.
-__device__ __forceinline__ int reserve(int* cnt, int total, int limit) {
-    int cur = *reinterpret_cast<volatile int*>(cnt);
-    while (true) {
-        if (cur + total > limit) return -1;
-        const int prev = atomicCAS(cnt, cur, cur + total);
-        if (prev == cur) return cur;
-        cur = prev;
+// Current bound / raise it (thread 0 inside a collective).
+template <class Key>
+__device__ __forceinline__ E32 bound_get(const CtaState<E32, Key>& st) { return E32{st.tau_w}; }
+template <class Key>
+__device__ __forceinline__ E64 bound_get(const CtaState<E64, Key>& st) { return st.tau; }
+template <class Key, bool MIN>
+__device__ __forceinline__ void bound_set(CtaState<E32, Key>* st, E32 t) {
+    if (t.v > st->tau_w) st->tau_w = t.v;
+}
+template <class Key, bool MIN>
+__device__ __forceinline__ void bound_set(CtaState<E64, Key>* st, E64 t) {
+    if (better(t, st->tau)) {
+        st->tau = t;
+        st->par = make_par<Key, MIN>(t);
     }
 }
+// The bound a consumer uses for one tile (changes only inside collectives).
+template <class Key, bool MIN>
+__device__ __forceinline__ Par<E32, Key> load_par(const CtaState<E32, Key>& st) {
+    return make_par<Key, MIN>(E32{st.tau_w});
+}
+template <class Key, bool MIN>
+__device__ __forceinline__ Par<E64, Key> load_par(const CtaState<E64, Key>& st) {
+    return st.par;
+}
 
-// Warp-aggregated append of this thread's kept entries ("computes a prefix sum
-// and then writes it out into a shared memory buffer").  Returns the buffer count
-// before this warp's entries, or -1 if they did not fit (nothing written).
+// Reserve `total` buffer entries (lane 31 of a warp): one atomicAdd; a reservation
+// that overshoots `limit` is undone and reported as -1.  Successful reservations are
+// always contiguous from 0 (a failed one leaves the counter above the limit until its
+// undo, so no success can start above it).
+__device__ __forceinline__ int reserve(int* cnt, int total, int limit) {
+    const int old = atomicAdd(cnt, total);
+    if (old + total <= limit) return old;
+    atomicSub(cnt, total);
+    return -1;
+}
+
+// Warp-aggregated append of ITEMS candidate entries per thread (mask = which).
+// Returns the count before this warp's entries, or -1 if they did not fit.
 template <class E, int ITEMS>
 __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&ents)[ITEMS],
-                                      uint32_t mask, int K, int* after) {
+                                      uint32_t mask, int K, int limit) {
     const int lane = threadIdx.x & 31;
     const int cnt = __popc(mask);
     int incl = cnt;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
-        int y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+        const int y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
         if (lane >= o) incl += y;
     }
     const int total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+    if (total == 0) return 0;
     int old = 0;
-    if (lane == 31 && total > 0) old = reserve(s_cnt, total, kCap - K);
+    if (lane == 31) old = reserve(s_cnt, total, limit);
     old = __shfl_sync(0xFFFFFFFFu, old, 31);
-    *after = old + total;
     if (old < 0) return -1;
     int w = K + old + incl - cnt;
 #pragma unroll
@@ -248,45 +301,174 @@ __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&
     return old;
 }
 
-// Collective flush (consumers): bitonic top-K of [run | survivors | padding]; updates
-// the CTA bound and publishes it.  Entry: barrier-consistent; exit: same.
-template <class Key, bool MIN>
-__device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
-                      CtaState<typename KeyTraits<Key>::E, Key>* st, WsHeader* hdr, int k,
-                      int K) {
-    using E = typename KeyTraits<Key>::E;
-    const int cnt = st->cnt;
-    int P = next_pow2_i(K + cnt);
-    if (P < 2 * K) P = 2 * K;
-    for (int i = K + cnt + threadIdx.x; i < P; i += kNC) buf.st(i, E::sentinel());
+// Debug counters (whole-launch totals), read with topk_debug_stats():
+// [0] flushes, [1] survivors flushed, [2] flush cycles (thread 0), [3] deferrals,
+// [4] tiles consumed, [5] refreshes.  Only rare paths touch them.
+__device__ unsigned long long g_stats[8];
+
+// Debug timeline: per CTA up to 62 (event << 56 | globaltimer ns) stamps written by
+// consumer thread 0 (events: 1 start, 2 flush begin, 3 flush end, 4 stream end,
+// 5 tail begin, 6 end, 7 refresh); g_trace[c][0] = count.  Enabled by g_trace_on.
+constexpr int kTraceCtas = 160, kTraceLen = 64;
+__device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
+__device__ int g_trace_on;
+__device__ __forceinline__ void trace(int ev) {
+    if (!g_trace_on || blockIdx.x >= kTraceCtas) return;
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    unsigned long long* row = g_trace[blockIdx.x];
+    const unsigned long long n = row[0];
+    if (n + 1 < kTraceLen) {
+        row[n + 1] = (static_cast<unsigned long long>(ev) << 56) | (t & 0x00FFFFFFFFFFFFFFull);
+        row[0] = n + 1;
+    }
+}
+
+// Everything a collective needs besides the buffer.
+struct Ctx {
+    WsHeader* hdr;
+    unsigned long long* pub;      // global [kPubRows][gmax]
+    unsigned long long* scratch;  // shared [J][G]
+    int k, K;
+    int G, gmax, J;
+    bool filter;
+};
+
+// Rank bound over scratch[J][G] (0 = missing sample): for row j the t-th largest word,
+// t = ceil(k / 2^j) <= G.  Collective (consumers); st->best[] receives one word per
+// row.  Entry: scratch filled and barrier passed; exit: after a barrier.
+template <class E, class Key>
+__device__ void rank_rows(CtaState<E, Key>* st, const Ctx& cx) {
+    if (threadIdx.x < kPubRows) st->best[threadIdx.x] = 0ull;
     CSync::sync();
-    bitonic_topk_smem<E, kNC, CSync>(buf, P, K);
-    if (threadIdx.x == 0) {
-        st->cnt = 0;
-        const E kth = buf.ld(k - 1);
-        if (!kth.is_sentinel()) {
-            tau_publish(hdr, kth);
-            if (better(kth, st->tau)) {
-                volatile uint32_t* ver = &st->tau_ver;
-                *ver = *ver + 1u;  // odd: writing
-                __threadfence_block();
-                st->tau = kth;
-                __threadfence_block();
-                *ver = *ver + 1u;
-            }
-        }
+    const int JG = cx.J * cx.G;
+    for (int q = threadIdx.x; q < JG; q += kNC) {
+        const int ji = q / cx.G;
+        const int t = (cx.k + (1 << ji) - 1) >> ji;
+        const unsigned long long v = cx.scratch[q];
+        if (t > cx.G || v == 0ull) continue;
+        const unsigned long long* row = cx.scratch + ji * cx.G;
+        int rank = 0;
+        for (int c2 = 0; c2 < cx.G; ++c2) rank += row[c2] > v ? 1 : 0;
+        if (rank == t - 1) st->best[ji] = v;  // unique: samples are distinct entries
     }
     CSync::sync();
 }
 
-// Consumer work on one tile held in shared memory: fast test, exact test, append.
-// Returns the append result (-1 = did not fit) and sets *vote if a flush is due.
+// Load every CTA's published samples into shared scratch (stale values are smaller,
+// still valid).
+__device__ __forceinline__ void load_pub(const Ctx& cx) {
+    const int JG = cx.J * cx.G;
+    for (int q = threadIdx.x; q < JG; q += kNC) {
+        const int ji = q / cx.G, cc = q % cx.G;
+        cx.scratch[q] = ld_relaxed_u64(
+            reinterpret_cast<const uint64_t*>(cx.pub + static_cast<size_t>(ji) * cx.gmax + cc));
+    }
+}
+
+// Fold st->best[] (and tau_g, and the run's own k-th best) into the CTA bound.
+template <class Key, bool MIN>
+__device__ __forceinline__ void fold_bounds(CtaState<typename KeyTraits<Key>::E, Key>* st,
+                                            const Ctx& cx, typename KeyTraits<Key>::E own) {
+    using E = typename KeyTraits<Key>::E;
+    E tau = bound_get(*st);
+    if (!own.is_sentinel() && better(own, tau)) tau = own;
+    const E tg =
+        from_bound_word<E>(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&cx.hdr->tau_g)));
+    if (better(tg, tau)) tau = tg;
+    for (int ji = 0; ji < cx.J; ++ji) {
+        const E b = from_bound_word<E>(st->best[ji]);
+        if (st->best[ji] != 0ull && better(b, tau)) tau = b;
+    }
+    bound_set<Key, MIN>(st, tau);
+}
+
+enum FlushMode { kFlushStream = 0, kFlushFinal = 1 };
+
+// Collective flush (consumers): bitonic top-K of [run | survivors | padding].
+//   stream mode: publish the run's samples and k-th best, and -- except for the very
+//   first flush, when no other CTA has published yet -- raise the bound with the rank
+//   bound over all CTAs' samples;  final mode: the network only.
+// Entry: barrier-consistent; exit: same.
+template <class Key, bool MIN>
+__device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
+                      CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx& cx,
+                      FlushMode mode) {
+    using E = typename KeyTraits<Key>::E;
+    const int k = cx.k, K = cx.K;
+    const int cnt = st->cnt;
+    if (threadIdx.x == 0) trace(2);
+    const long long t0 = clock64();
+    int P = next_pow2_i(K + cnt);
+    if (P < 2 * K) P = 2 * K;
+    for (int i = K + cnt + threadIdx.x; i < P; i += kNC) buf.st(i, E::sentinel());
+    CSync::sync();
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (K <= 256)
+        wnet_topk<E, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
+    else
+        bitonic_topk_smem<E, kNC, CSync>(buf, P, K);
+    const E kth = buf.ld(k - 1);
+    const bool publish = mode == kFlushStream && cx.filter;
+    const bool ranks = publish && st->nflush > 0;
+    if (publish) {
+        const int c = static_cast<int>(blockIdx.x);
+        if (threadIdx.x < cx.J) {
+            const E e = buf.ld((1 << threadIdx.x) - 1);
+            if (!e.is_sentinel())
+                st_relaxed_u64(cx.pub + static_cast<size_t>(threadIdx.x) * cx.gmax + c,
+                               bound_word(e));
+        }
+        if (threadIdx.x == 0 && !kth.is_sentinel()) tau_publish(cx.hdr, kth);
+        if (ranks) {
+            load_pub(cx);
+            CSync::sync();
+            rank_rows(st, cx);
+        }
+    }
+    if (threadIdx.x == 0) {
+        atomicAdd(&g_stats[0], 1ull);
+        atomicAdd(&g_stats[1], static_cast<unsigned long long>(cnt));
+        atomicAdd(&g_stats[2], static_cast<unsigned long long>(clock64() - t0));
+        st->cnt = 0;
+        st->nflush += 1;
+        if (!ranks)
+            for (int ji = 0; ji < kPubRows; ++ji) st->best[ji] = 0ull;
+        if (cx.filter) fold_bounds<Key, MIN>(st, cx, kth);
+        st->req = 0;
+        trace(3);
+    }
+    CSync::sync();
+}
+
+// Collective bound refresh (no flush): rank bound over all CTAs' published samples.
+template <class Key, bool MIN>
+__device__ void refresh(CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx& cx) {
+    using E = typename KeyTraits<Key>::E;
+    load_pub(cx);
+    CSync::sync();
+    rank_rows(st, cx);
+    if (threadIdx.x == 0) {
+        atomicAdd(&g_stats[5], 1ull);
+        fold_bounds<Key, MIN>(st, cx, E::sentinel());
+        st->req = 0;
+        trace(7);
+    }
+    CSync::sync();
+}
+
+// Consumer work on one tile held in shared memory.
+//   fast pass: one compare per key against the threshold key, OR-reduced per warp --
+//              the only work for the vast majority of tiles;
+//   slow pass (some lane passed): per-key mask, exact entry test on the passing keys
+//              (re-read from shared memory), warp prefix sum, one reservation, writes.
+// Returns the buffer count before this warp's entries, or -1 if they did not fit.
 template <class Key, bool MIN, bool FILTER>
 __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
                                             const Par<typename KeyTraits<Key>::E, Key>& pr,
                                             uint32_t tlen, uint32_t lbase,
                                             const SBuf<typename KeyTraits<Key>::E>& buf,
-                                            int* s_cnt, int K, int flush_soft, int* vote) {
+                                            int* s_cnt, int K, int limit) {
     using KT = KeyTraits<Key>;
     using E = typename KT::E;
     using Vec = typename KT::Vec;
@@ -296,27 +478,45 @@ __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
     constexpr int ITEMS = C::kItems;
     constexpr int TK = C::kTileKeys;
     const int tid = threadIdx.x;
+    const int lane = tid & 31;
 
     const Vec* sv = reinterpret_cast<const Vec*>(slot_data);
+    const Key* sk = reinterpret_cast<const Key*>(slot_data);
     Vec v[VPT];
 #pragma unroll
     for (int j = 0; j < VPT; ++j) v[j] = sv[tid + j * kNC];
 
+    const bool all = !FILTER || !pr.active;
+    const bool strict = lbase > pr.strict_after;
+    bool anyp = all;
+    if (!all) {
+        if (strict) {
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                anyp |= KT::template fast<MIN, true>(vget(v[q / VEC], q % VEC), pr.t);
+        } else {
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                anyp |= KT::template fast<MIN, false>(vget(v[q / VEC], q % VEC), pr.t);
+        }
+    }
+    if (!__any_sync(0xFFFFFFFFu, anyp)) return 0;
+
     uint32_t mask = 0;
-    if (!FILTER || !pr.active) {
+    if (all) {
         mask = (ITEMS >= 32) ? 0xFFFFFFFFu : ((1u << ITEMS) - 1u);
-    } else if (lbase > pr.strict_after) {
+    } else if (anyp) {
+        if (strict) {
 #pragma unroll
-        for (int q = 0; q < ITEMS; ++q)
-            mask |= static_cast<uint32_t>(
-                        KT::template fast<MIN, true>(vget(v[q / VEC], q % VEC), pr.t))
-                    << q;
-    } else {
+            for (int q = 0; q < ITEMS; ++q)
+                mask |= static_cast<uint32_t>(
+                            KT::template fast<MIN, true>(vget(v[q / VEC], q % VEC), pr.t)) << q;
+        } else {
 #pragma unroll
-        for (int q = 0; q < ITEMS; ++q)
-            mask |= static_cast<uint32_t>(
-                        KT::template fast<MIN, false>(vget(v[q / VEC], q % VEC), pr.t))
-                    << q;
+            for (int q = 0; q < ITEMS; ++q)
+                mask |= static_cast<uint32_t>(
+                            KT::template fast<MIN, false>(vget(v[q / VEC], q % VEC), pr.t)) << q;
+        }
     }
     if (tlen < static_cast<uint32_t>(TK)) {
 #pragma unroll
@@ -325,22 +525,38 @@ __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
             if (pos >= tlen) mask &= ~(1u << q);
         }
     }
-    *vote = 0;
-    if (!__any_sync(0xFFFFFFFFu, mask != 0u)) return 0;
-    E ents[ITEMS];
-#pragma unroll
-    for (int q = 0; q < ITEMS; ++q) {
-        ents[q] = E::sentinel();
-        if ((mask >> q) & 1u) {
-            const uint32_t pos = static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + q % VEC);
-            const E e = E::make(KT::template code<MIN>(vget(v[q / VEC], q % VEC)), lbase + pos);
-            ents[q] = e;
-            if (FILTER && pr.active && !better(e, pr.tau)) mask &= ~(1u << q);
+    auto pos_of = [&](int q) -> uint32_t {
+        return static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
+    };
+    uint32_t keep = mask;
+    if (FILTER && pr.active) {  // exact entry test (R1 order) on the passing keys
+        keep = 0;
+        for (uint32_t m = mask; m; m &= m - 1u) {
+            const int q = __ffs(m) - 1;
+            const uint32_t pos = pos_of(q);
+            const E e = E::make(KT::template code<MIN>(sk[pos]), lbase + pos);
+            if (better(e, pr.tau)) keep |= 1u << q;
         }
     }
-    int after = 0;
-    const int old = append<E, ITEMS>(buf, s_cnt, ents, mask, K, &after);
-    *vote = (old < 0 || after > flush_soft) ? 1 : 0;
+    const int cnt = __popc(keep);
+    int incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+        if (lane >= o) incl += y;
+    }
+    const int total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+    if (total == 0) return 0;
+    int old = 0;
+    if (lane == 31) old = reserve(s_cnt, total, limit);
+    old = __shfl_sync(0xFFFFFFFFu, old, 31);
+    if (old < 0) return -1;
+    int w = K + old + incl - cnt;
+    for (uint32_t m = keep; m; m &= m - 1u) {
+        const int q = __ffs(m) - 1;
+        const uint32_t pos = pos_of(q);
+        buf.st(w++, E::make(KT::template code<MIN>(sk[pos]), lbase + pos));
+    }
     return old;
 }
 
@@ -350,6 +566,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     using E = typename KT::E;
     using C = Cfg<Key>;
     constexpr int TK = C::kTileKeys;
+    constexpr int kStages = C::kStages;
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ CtaState<E, Key> st;
@@ -360,16 +577,27 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + static_cast<size_t>(kStages) * kTileBytes +
                                                  static_cast<size_t>(kCap) * SBuf<E>::kBytes);
     uint64_t* empty = full + kStages;
+    unsigned long long* scratch = reinterpret_cast<unsigned long long*>(empty + kStages);
 
     const int tid = threadIdx.x;
     const uint32_t G = gridDim.x;
     const uint32_t c = blockIdx.x;
     const int K = static_cast<int>(p.K);
     const int k = static_cast<int>(p.k);
-    const int flush_soft = kCap - K - 2048;
+    // Until a bound exists, keep the buffer small so the first flush is cheap.
+    const int boot_limit = FILTER ? (K > 1024 ? K : 1024) : kCap - K;
     const Key* keys = static_cast<const Key*>(p.keys);
     WsHeader* hdr = reinterpret_cast<WsHeader*>(p.ws);
-    const uint32_t my_tiles = c < p.ntiles ? (p.ntiles - c + G - 1) / G : 0u;
+    Ctx cx;
+    cx.hdr = hdr;
+    cx.pub = reinterpret_cast<unsigned long long*>(p.ws + ws_pub_offset());
+    cx.scratch = scratch;
+    cx.k = k;
+    cx.K = K;
+    cx.G = static_cast<int>(G);
+    cx.gmax = static_cast<int>(p.gmax);
+    cx.J = static_cast<int>(p.J);
+    cx.filter = FILTER;
 
     for (int i = tid; i < K; i += kNT) buf.st(i, E::sentinel());
     if (tid == 0) {
@@ -379,8 +607,11 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         }
         fence_mbar_init();
         st.cnt = 0;
-        st.tau_ver = 0;
+        st.req = 0;
+        st.nflush = 0;
+        st.tau_w = 0ull;
         st.tau = E::sentinel();
+        st.par = make_par<Key, MIN>(E::sentinel());
     }
     // Extras: the unaligned head and the sub-16-byte tail, appended by CTA 0.
     if (c == 0) {
@@ -396,83 +627,114 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     __syncthreads();
 
     if (tid >= kNC) {
-        // ---------------- producer warp (one lane) ----------------
+        // ---------------- producer warp (lane 0) ----------------
         if (tid != kNC) return;
         const Key* body = keys + p.head;
         const uint64_t policy = l2_evict_first_policy();
-        uint64_t tg_next = FILTER ? tau_load_raw(hdr) : 0ull;
-        for (uint32_t s = 0; s < my_tiles; ++s) {
+        const uint32_t blk = p.blk;
+        const uint32_t nclaim = p.nwaves * p.wave * blk;
+        uint32_t claim = 0, left = 0;
+        uint32_t pending = atomicAdd(&hdr->next_tile, blk);
+#pragma unroll 1
+        for (uint32_t s = 0;; ++s) {
             const int slot = static_cast<int>(s % kStages);
+            uint32_t tile = kEndTile;
+            while (true) {
+                if (left == 0) {
+                    claim = pending;  // consumes the outstanding claim
+                    left = blk;
+                    if (claim >= nclaim) break;
+                    pending = atomicAdd(&hdr->next_tile, blk);
+                }
+                const uint32_t i = claim++;
+                --left;
+                // claim i -> block b = (wave, position); waves permuted, the blocks of a
+                // wave adjacent; tiles of a block in address order
+                const uint32_t b = i / blk;
+                const uint32_t pb =
+                    feistel_perm(b / p.wave, p.nwaves, p.perm_h) * p.wave + b % p.wave;
+                const uint32_t t = pb * blk + i % blk;
+                if (t < p.ntiles) {
+                    tile = t;
+                    break;
+                }
+            }
             if (s >= static_cast<uint32_t>(kStages))
                 mbar_wait(&empty[slot], ((s / kStages) - 1u) & 1u);
-            const uint32_t tile = tile_of(c + s * G, p.ntiles, p.perm_h);
+            st.tile[slot] = tile;
+            if (tile == kEndTile) {
+                mbar_arrive(&full[slot]);  // no bytes: the consumers see kEndTile
+                return;
+            }
             const uint64_t lo = static_cast<uint64_t>(tile) * TK;
             const uint64_t len = min(static_cast<uint64_t>(TK), p.body_n - lo);
             const uint32_t bytes = static_cast<uint32_t>(len * sizeof(Key));
-            tma_load_1d(ring + static_cast<size_t>(slot) * kTileBytes, body + lo, bytes,
-                        &full[slot], policy);
-            SlotMeta<E, Key> m;
-            m.tlen = static_cast<uint32_t>(len);
-            m.lbase = static_cast<uint32_t>(p.head + lo);
-            if (FILTER) {
-                const E tg = tau_from_raw<E>(tg_next);
-                tg_next = tau_load_raw(hdr);  // prefetch for the next tile
-                E tl;
-                uint32_t v1, v2;
-                do {
-                    v1 = *reinterpret_cast<volatile uint32_t*>(&st.tau_ver);
-                    __threadfence_block();
-                    tl = load_volatile(&st.tau);
-                    __threadfence_block();
-                    v2 = *reinterpret_cast<volatile uint32_t*>(&st.tau_ver);
-                } while (v1 != v2 || (v1 & 1u));
-                m.par = make_par<Key, MIN>(better(tg, tl) ? tg : tl);
-            } else {
-                m.par = make_par<Key, MIN>(E::sentinel());
-            }
-            st.meta[slot] = m;
-            mbar_arrive_expect_tx(&full[slot], bytes);  // release: meta visible with data
+            tma_load_1d(ring + static_cast<size_t>(slot) * kTileBytes, body + lo, bytes, &full[slot],
+                        policy);
+            mbar_arrive_expect_tx(&full[slot], bytes);  // release: tile id visible
         }
-        return;
     }
 
     // ---------------- consumer warps ----------------
     const int lane = tid & 31;
-    for (uint32_t s = 0; s < my_tiles; ++s) {
+    if (tid == 0) trace(1);
+    auto pending_req = [&]() -> bool { return *reinterpret_cast<volatile int*>(&st.req) != 0; };
+    // Body of a collective, entered by all consumer warps after one OR-barrier.
+    auto collective = [&]() {
+        if (st.req & kReqFlush)
+            flush<Key, MIN>(buf, &st, cx, kFlushStream);
+        else
+            refresh<Key, MIN>(&st, cx);
+    };
+    uint32_t ntiles_done = 0;
+#pragma unroll 1
+    for (uint32_t s = 0;; ++s) {
         const int slot = static_cast<int>(s % kStages);
-        mbar_wait(&full[slot], (s / kStages) & 1u);
-        const SlotMeta<E, Key> m = st.meta[slot];
-        const unsigned char* data = ring + static_cast<size_t>(slot) * kTileBytes;
-        int vote;
-        int r = consume_tile<Key, MIN, FILTER>(data, m.par, m.tlen, m.lbase, buf, &st.cnt, K,
-                                               flush_soft, &vote);
-        bool deferred = r < 0;
-        if (!deferred) {
-            __syncwarp();
-            if (lane == 0) mbar_arrive(&empty[slot]);
-        }
-        while (cbar_or(vote != 0)) {
-            flush<Key, MIN>(buf, &st, hdr, k, K);
-            vote = 0;
-            if (deferred) {  // redo this warp's part of the tile with the new bound
-                const E tau = better(st.tau, m.par.tau) ? st.tau : m.par.tau;
-                const Par<E, Key> pr = make_par<Key, MIN>(tau);
-                r = consume_tile<Key, MIN, FILTER>(data, pr, m.tlen, m.lbase, buf, &st.cnt, K,
-                                                   flush_soft, &vote);
-                deferred = r < 0;
-                if (!deferred) {
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&empty[slot]);
-                }
+        const uint32_t parity = (s / kStages) & 1u;
+        while (true) {
+            if (pending_req()) {
+                cbar_or(true);
+                collective();
+                continue;
             }
+            if (mbar_try_wait(&full[slot], parity)) break;
         }
+        const uint32_t tile = st.tile[slot];
+        if (tile == kEndTile) break;
+        ++ntiles_done;
+        const uint64_t tlo = static_cast<uint64_t>(tile) * TK;
+        const uint32_t tlen = static_cast<uint32_t>(min(static_cast<uint64_t>(TK), p.body_n - tlo));
+        const uint32_t lbase = static_cast<uint32_t>(p.head + tlo);
+        const unsigned char* data = ring + static_cast<size_t>(slot) * kTileBytes;
+        Par<E, Key> pr = load_par<Key, MIN>(st);
+        int r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, K,
+                                               pr.active ? kCap - K : boot_limit);
+        while (r < 0) {  // did not fit: flush, then redo with the new bound
+            if (lane == 0) {
+                atomicAdd(&g_stats[3], 1ull);
+                atomicOr(&st.req, kReqFlush);
+            }
+            __syncwarp();
+            cbar_or(true);
+            collective();
+            pr = load_par<Key, MIN>(st);
+            r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, K,
+                                               pr.active ? kCap - K : boot_limit);
+        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[slot]);
+        // Once every CTA has had time to publish its first run, pull the rank bound.
+        if (FILTER && G > 1 && tid == 0 && s == TOPK_REFRESH_AT) atomicOr(&st.req, kReqRefresh);
     }
-    CSync::sync();
-    if (st.cnt > 0) flush<Key, MIN>(buf, &st, hdr, k, K);
+    // Drain: serve requests of warps still streaming, until all are done.
+    while (cbar_or(pending_req())) collective();
+    if (tid == 0) trace(4);
+    if (tid == 0) atomicAdd(&g_stats[4], static_cast<unsigned long long>(ntiles_done));
+    if (st.cnt > 0) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
 
     // ---- hand the CTA's top-k to the reduction (last CTA to arrive) ----
     GBuf<E> cand;
-    cand.init(p.ws + sizeof(WsHeader), static_cast<size_t>(G) * k);
+    cand.init(p.ws + ws_cand_offset(p.gmax), static_cast<size_t>(G) * k);
     if (G > 1) {
         for (int j = tid; j < k; j += kNC) cand.st(static_cast<size_t>(c) * k + j, buf.ld(j));
         __threadfence();
@@ -481,46 +743,78 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         CSync::sync();
         if (!st.last) return;
         __threadfence();
-        // Candidates of every other CTA that can still be in the top-k: e >= tau_g
-        // (tau_g is some CTA's k-th best, so anything worse has k better entries).
-        const E tg = tau_from_raw<E>(tau_load_raw(hdr));
-        const size_t total = static_cast<size_t>(G) * k;
-        constexpr int CI = 8;  // entries per thread per chunk
-        constexpr int CH = CI * kNC;
-        for (size_t q0 = 0; q0 < total; q0 += CH) {
-            E ents[CI];
-            uint32_t mask = 0;
-#pragma unroll
-            for (int r = 0; r < CI; ++r) {
-                const size_t q = q0 + tid + static_cast<size_t>(r) * kNC;
-                ents[r] = E::sentinel();
-                if (q < total && q / k != c) {
-                    const E e = cand.ld(q);
-                    if (!e.is_sentinel() && !better(tg, e)) {
-                        ents[r] = e;
-                        mask |= 1u << r;
-                    }
-                }
-            }
-            bool deferred = true;
-            while (true) {
-                int vote = 0;
-                if (deferred) {
-                    int after = 0;
-                    if (__any_sync(0xFFFFFFFFu, mask != 0u)) {
-                        const int old = append<E, CI>(buf, &st.cnt, ents, mask, K, &after);
-                        deferred = old < 0;
-                        vote = deferred ? 1 : 0;
-                    } else {
-                        deferred = false;
-                    }
-                }
-                if (!cbar_or(vote != 0)) break;
-                flush<Key, MIN>(buf, &st, hdr, k, K);
-            }
+        if (tid == 0) trace(5);
+        // (1) Rank bound over the final runs (tail form of the flush bound): row j holds
+        // each run's 2^j-th best; the t-th largest (t = ceil(k / 2^j) <= G) bounds the
+        // global k-th best.  All loads in one parallel pass.
+        for (int q = tid; q < cx.J * cx.G; q += kNC) {
+            const int ji = q / cx.G, cc = q % cx.G;
+            scratch[q] = bound_word(cand.ld(static_cast<size_t>(cc) * k + (1u << ji) - 1u));
         }
         CSync::sync();
-        if (st.cnt > 0) flush<Key, MIN>(buf, &st, hdr, k, K);
+        rank_rows(&st, cx);
+        if (tid == 0) {
+            E tb = from_bound_word<E>(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&hdr->tau_g)));
+            for (int ji = 0; ji < cx.J; ++ji) {
+                const E b = from_bound_word<E>(st.best[ji]);
+                if (st.best[ji] != 0ull && better(b, tb)) tb = b;
+            }
+            st.tau = tb;
+            st.cnt = 0;
+        }
+        CSync::sync();
+        const E tb = st.tau;
+        // (2) Every run is sorted best first, so only a prefix can be >= tb: append the
+        // qualifying entries of the first min(k, 32) of every other run (one parallel
+        // pass), then the rest of the runs whose 32nd entry still qualified (rare).
+        const int kk = k < 32 ? k : 32;
+        __shared__ unsigned int s_more[(kGMax + 31) / 32];
+        for (int q = tid; q < (kGMax + 31) / 32; q += kNC) s_more[q] = 0u;
+        CSync::sync();
+        constexpr int CI = 8;
+        for (int phase = 0; phase < 2; ++phase) {
+            const int lo = phase == 0 ? 0 : kk;
+            const int span = phase == 0 ? kk : k - kk;
+            if (span <= 0) break;
+            const int total = cx.G * span;
+            for (int q0 = 0; q0 < total; q0 += CI * kNC) {
+                E ents[CI];
+                uint32_t mask = 0;
+#pragma unroll
+                for (int r = 0; r < CI; ++r) {
+                    const int q = q0 + tid + r * kNC;
+                    ents[r] = E::sentinel();
+                    if (q >= total) continue;
+                    const int cc = q / span, j = lo + q % span;
+                    if (cc == static_cast<int>(c)) continue;
+                    if (phase == 1 && !((s_more[cc >> 5] >> (cc & 31)) & 1u)) continue;
+                    const E e = cand.ld(static_cast<size_t>(cc) * k + j);
+                    if (!e.is_sentinel() && !better(tb, e)) {
+                        ents[r] = e;
+                        mask |= 1u << r;
+                        if (phase == 0 && j == kk - 1 && kk < k)
+                            atomicOr(&s_more[cc >> 5], 1u << (cc & 31));
+                    }
+                }
+                bool todo = true;
+                while (true) {
+                    int vote = 0;
+                    if (todo) {
+                        if (__any_sync(0xFFFFFFFFu, mask != 0u)) {
+                            const int old = append<E, CI>(buf, &st.cnt, ents, mask, K, kCap - K);
+                            todo = old < 0;
+                            vote = todo ? 1 : 0;
+                        } else {
+                            todo = false;
+                        }
+                    }
+                    if (!cbar_or(vote != 0)) break;
+                    flush<Key, MIN>(buf, &st, cx, kFlushFinal);
+                }
+            }
+            CSync::sync();
+        }
+        if (st.cnt > 0) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
     }
     // ---- finalize: best first, original key bits, global index, payload ----
     for (int j = tid; j < k; j += kNC) {
@@ -530,17 +824,22 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = keys[row];
         if (p.out_payload) p.out_payload[j] = p.payload[row];
     }
-    if (tid == 0) {  // leave the workspace zeroed for the next call
+    if (tid == 0) trace(6);
+    // leave the workspace zeroed for the next call (all other CTAs are done)
+    for (int q = tid; q < kPubRows * static_cast<int>(G); q += kNC)
+        cx.pub[static_cast<size_t>(q / G) * p.gmax + q % G] = 0ull;
+    if (tid == 0) {
         hdr->tau_g = 0ull;
         hdr->ticket = 0u;
+        hdr->next_tile = 0u;
     }
 }
 
 template <class Key>
 constexpr size_t select_smem_bytes() {
-    return static_cast<size_t>(kStages) * kTileBytes +
+    return static_cast<size_t>(Cfg<Key>::kStages) * kTileBytes +
            static_cast<size_t>(kCap) * SBuf<typename KeyTraits<Key>::E>::kBytes +
-           static_cast<size_t>(2 * kStages) * 8;
+           static_cast<size_t>(2 * Cfg<Key>::kStages) * 8 + static_cast<size_t>(kScratch) * 8;
 }
 
 }  // namespace topk

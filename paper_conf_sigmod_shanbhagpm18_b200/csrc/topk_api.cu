@@ -5,9 +5,12 @@
 
 #include <atomic>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 
 #include "merge.cuh"
+#include "probe.cuh"
+#include "netbench.cuh"
 #include "select.cuh"
 #include "topk.h"
 
@@ -124,7 +127,8 @@ size_t topk_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k) {
     if (!valid_dtype(dtype) || n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return 0;
     int sms = 0, major = 0;
     if (!device_info(&sms, &major)) return 0;
-    return align_up(sizeof(topk::WsHeader) + static_cast<size_t>(sms) * k * entry_bytes(dtype),
+    return align_up(topk::ws_cand_offset(static_cast<uint32_t>(sms)) +
+                        static_cast<size_t>(sms) * k * entry_bytes(dtype),
                     256);
 }
 
@@ -149,7 +153,7 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
     if (n > kMaxLaunchN) return TOPK_ERR_UNSUPPORTED;  // chunked path: see DESIGN.md §9
     int sms = 0, major = 0;
     if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
-    if (major != 10) return TOPK_ERR_UNSUPPORTED;
+    if (major != 10 || sms > topk::kGMax) return TOPK_ERR_UNSUPPORTED;
     const size_t need = topk_workspace_bytes(dtype, n, k);
     if (!ws || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws) % 256)) return TOPK_ERR_WORKSPACE;
 
@@ -173,11 +177,36 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
     p.ntiles = static_cast<uint32_t>(ntiles);
     p.k = k;
     p.K = next_pow2_u32(k);
-    // Tile permutation half-width: 2h bits cover ntiles.
+    // Work blocks (tiles claimed together) and their permutation (2h bits cover them).
+    p.blk = ntiles >= 16ull * static_cast<uint64_t>(sms) ? 8u : 1u;
+    static const int blk_env = [] {
+        const char* v = std::getenv("TOPK_BLOCK");
+        return v ? std::atoi(v) : 0;
+    }();
+    if (blk_env > 0) p.blk = static_cast<uint32_t>(blk_env);
+    p.nblocks = static_cast<uint32_t>((ntiles + p.blk - 1) / p.blk);
+    static const int wave_env = [] {
+        const char* v = std::getenv("TOPK_WAVE");
+        return v ? std::atoi(v) : 0;
+    }();
+    // default: one block per SM per wave -- all SMs stream one address window at a
+    // time (DRAM row locality), waves in pseudo-random order (robust to sorted input)
+    p.wave = wave_env > 0 ? static_cast<uint32_t>(wave_env) : static_cast<uint32_t>(sms);
+    if (false) p.wave = wave_env > 0 ? static_cast<uint32_t>(wave_env) : 1u;
+    p.nwaves = (p.nblocks + p.wave - 1) / p.wave;
     uint32_t bits = 0;
-    while ((1ull << bits) < ntiles) ++bits;
-    p.perm_h = ntiles > 1 ? (bits + 1) / 2 : 0;
+    while ((1ull << bits) < p.nwaves) ++bits;
+    p.perm_h = p.nwaves > 1 ? (bits + 1) / 2 : 0;
+    static const int perm_env = [] {
+        const char* v = std::getenv("TOPK_PERM");
+        return v ? std::atoi(v) : 1;
+    }();
+    if (!perm_env) p.perm_h = 0;
     const int grid = static_cast<int>(ntiles == 0 ? 1 : (ntiles < (uint64_t)sms ? ntiles : sms));
+    p.gmax = static_cast<uint32_t>(sms);
+    // Published samples: the 2^j-th best of each run for 2^j <= k (select.cuh flush).
+    p.J = 0;
+    while (p.J < static_cast<uint32_t>(topk::kPubRows) && (1u << p.J) <= k) ++p.J;
 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
@@ -266,6 +295,77 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
         default: e = dispatch_merge<double>(p, mn, st); break;
     }
     return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+}
+
+/* Debug (not in topk.h's stable surface): read / reset the device counters of
+ * select_kernel (flushes, survivors flushed, flush cycles, deferrals, tiles). */
+int topk_debug_stats(uint64_t* host8, int reset) {
+    if (cudaMemcpyFromSymbol(host8, topk::g_stats, sizeof(unsigned long long) * 8) != cudaSuccess)
+        return -1;
+    if (reset) {
+        unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (cudaMemcpyToSymbol(topk::g_stats, z, sizeof(z)) != cudaSuccess) return -1;
+    }
+    return 0;
+}
+
+topk_status_t topk_probe_read(const void* data, size_t bytes, int method, int grid, int tile,
+                              int stages, uint32_t* sink, void* stream) {
+    if (!data || !sink || bytes == 0 || (bytes % 16) || (reinterpret_cast<uintptr_t>(data) % 16))
+        return TOPK_ERR_INVALID_ARG;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    if (method == 0) {
+        const int g = grid > 0 ? grid : 4 * sms;
+        topk::probe_ldg_kernel<<<g, 512, 0, st>>>(static_cast<const uint4*>(data), bytes / 16,
+                                                  sink);
+    } else if (method == 1) {
+        if (tile <= 0 || (tile % 16) || stages <= 0) return TOPK_ERR_INVALID_ARG;
+        const size_t smem = static_cast<size_t>(tile) * stages + 16 * static_cast<size_t>(stages);
+        if (smem > 227 * 1024) return TOPK_ERR_INVALID_ARG;
+        if (cudaFuncSetAttribute(topk::probe_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 static_cast<int>(smem)) != cudaSuccess)
+            return TOPK_ERR_CUDA;
+        const int g = grid > 0 ? grid : sms;
+        topk::probe_tma_kernel<<<g, 512, smem, st>>>(static_cast<const unsigned char*>(data),
+                                                     bytes, tile, stages, sink);
+    } else {
+        return TOPK_ERR_INVALID_ARG;
+    }
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return cudaGetLastError() == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+}
+
+/* Debug: cycles of one flush network call on P entries (K = 2^L), measured in one CTA
+ * of 15 warps.  e64 selects 12-byte entries; smem_net the shared-memory network. */
+int topk_debug_netbench(int P, int L, int e64, int smem_net, int iters, uint64_t* host2) {
+    unsigned long long* d = nullptr;
+    if (cudaMalloc(&d, 16) != cudaSuccess) return -1;
+    const size_t smem = 4096 * 12;
+    if (e64) {
+        cudaFuncSetAttribute(topk::netbench_kernel<topk::E64, 15>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        topk::netbench_kernel<topk::E64, 15><<<1, 480, smem>>>(P, L, iters, smem_net, d);
+    } else {
+        cudaFuncSetAttribute(topk::netbench_kernel<topk::E32, 15>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        topk::netbench_kernel<topk::E32, 15><<<1, 480, smem>>>(P, L, iters, smem_net, d);
+    }
+    cudaError_t e = cudaMemcpy(host2, d, 16, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    return e == cudaSuccess ? 0 : -1;
+}
+
+/* Debug timeline (see select.cuh g_trace): enable=1 clears and enables, 0 disables;
+ * copies kTraceCtas x kTraceLen u64 to host (may be NULL). */
+int topk_debug_trace(int enable, uint64_t* host) {
+    if (host && cudaMemcpyFromSymbol(host, topk::g_trace, sizeof(topk::g_trace)) != cudaSuccess)
+        return -1;
+    static unsigned long long zero[topk::kTraceCtas][topk::kTraceLen];
+    if (cudaMemcpyToSymbol(topk::g_trace, zero, sizeof(zero)) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(topk::g_trace_on, &enable, sizeof(int)) != cudaSuccess) return -1;
+    return 0;
 }
 
 uint64_t topk_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }

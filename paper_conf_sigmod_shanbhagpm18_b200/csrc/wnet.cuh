@@ -1,0 +1,193 @@
+// wnet.cuh -- register/warp-shuffle form of the paper's operators for K <= 256.
+//
+// The paper fuses its operators into kernels whose steps run in shared memory
+// ("Operating in Shared Memory") and then combines several steps per thread
+// in registers ("Combining/Sequentializing Multiple Steps"; "elements per
+// thread B = 16").  On sm_100a the same idea is taken to the warp: a warp holds
+// R entries per lane in blocked layout (element e = lane * R + r), so a bitonic step
+// on element-index bit b is
+//   * b < log2 R : a compare-exchange between two registers of one thread, or
+//   * otherwise  : a warp shuffle with lane ^ (1 << (b - log2 R)) -- no shared memory.
+// Only the reduction rounds (merge + rebuild of pairs of runs held by different warps)
+// go through shared memory, one barrier pair per round.
+//
+// Step semantics are Alg. 4's generalised to any bit: element e is paired
+// with e ^ 2^b; blocks of 2^d elements alternate best-first / worst-first
+// (bit d of e == 0 -> best-first); the lower element of a pair in a best-first block
+// keeps the better entry.
+//
+// The step loops are NOT unrolled (only the per-register work is): a fully unrolled
+// K = 256 network is ~10^4 distinct instructions per flush and runs out of the
+// instruction cache.
+#pragma once
+#include "keys.cuh"
+
+namespace topk {
+
+template <class E>
+__device__ __forceinline__ E shfl_xor_e(const E& e, int m);
+template <>
+__device__ __forceinline__ E32 shfl_xor_e<E32>(const E32& e, int m) {
+    const uint32_t lo = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.v), m);
+    const uint32_t hi = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.v >> 32), m);
+    return E32{(static_cast<uint64_t>(hi) << 32) | lo};
+}
+template <>
+__device__ __forceinline__ E64 shfl_xor_e<E64>(const E64& e, int m) {
+    const uint32_t lo = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.c), m);
+    const uint32_t hi = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.c >> 32), m);
+    const uint32_t ni = __shfl_xor_sync(0xFFFFFFFFu, e.ni, m);
+    return E64{(static_cast<uint64_t>(hi) << 32) | lo, ni};
+}
+
+// Compare-exchange of two registers: afterwards a holds the better entry iff a_better.
+template <class E>
+__device__ __forceinline__ void cmpx(E& a, E& b, bool a_better) {
+    const bool sw = a_better == better(b, a);  // entries are distinct (or both sentinel)
+    const E ta = esel(sw, b, a);
+    const E tb = esel(sw, a, b);
+    a = ta;
+    b = tb;
+}
+
+template <int R>
+struct Log2 {
+    static constexpr int v = 1 + Log2<R / 2>::v;
+};
+template <>
+struct Log2<1> {
+    static constexpr int v = 0;
+};
+
+// Register step on bit B; wm bit r set <=> register r lies in a worst-first block.
+template <class E, int R, int B>
+__device__ __forceinline__ void reg_step(E (&x)[R], uint32_t wm) {
+#pragma unroll
+    for (int r = 0; r < R; ++r)
+        if ((r & (1 << B)) == 0) cmpx(x[r], x[r | (1 << B)], ((wm >> r) & 1u) == 0u);
+}
+
+// One bitonic step on element bit b with direction bit d (d > b); e0 = element index
+// of x[0] of this lane (chunk base + lane * R).
+template <class E, int R>
+__device__ __forceinline__ void wstep(E (&x)[R], int lane, uint32_t e0, int b, int d) {
+    constexpr int LR = Log2<R>::v;
+    if (b < LR) {
+        uint32_t wm;
+        if (d < LR) {
+            wm = 0;
+#pragma unroll
+            for (int r = 0; r < R; ++r) wm |= ((static_cast<uint32_t>(r) >> d) & 1u) << r;
+        } else {
+            wm = ((e0 >> d) & 1u) ? 0xFFFFFFFFu : 0u;
+        }
+        switch (b) {
+            case 0: reg_step<E, R, 0>(x, wm); break;
+            case 1: if constexpr (LR > 1) reg_step<E, R, 1>(x, wm); break;
+            case 2: if constexpr (LR > 2) reg_step<E, R, 2>(x, wm); break;
+            default: if constexpr (LR > 3) reg_step<E, R, 3>(x, wm); break;
+        }
+    } else {
+        const int m = 1 << (b - LR);
+        const bool lower = (lane & m) == 0;
+        const bool bf = ((e0 >> d) & 1u) == 0u;  // d > b >= LR: same for all r
+        const bool keep_better = lower == bf;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const E y = shfl_xor_e(x[r], m);
+            x[r] = esel(keep_better == better(y, x[r]), y, x[r]);
+        }
+    }
+}
+
+// Local sort (Alg. 2): runs of length 2^L alternating best-first / worst-first.
+template <class E, int R>
+__device__ __forceinline__ void wsort_runs(E (&x)[R], int lane, uint32_t e0, int L) {
+#pragma unroll 1
+    for (int s = 0; s < L; ++s)
+#pragma unroll 1
+        for (int b = s; b >= 0; --b) wstep<E, R>(x, lane, e0, b, s + 1);
+}
+
+// Rebuild (Alg. 4): steps L-1 .. 0 with direction bit L.
+template <class E, int R>
+__device__ __forceinline__ void wrebuild(E (&x)[R], int lane, uint32_t e0, int L) {
+#pragma unroll 1
+    for (int b = L - 1; b >= 0; --b) wstep<E, R>(x, lane, e0, b, L);
+}
+
+// Bitonic top-K (K = 2^L <= 256) of b[0..P), P a power of two, 2K <= P <= 4096, by
+// the NW warps of the calling group (warp index w, lane), all of which call this.
+// Result: b[0..K) best first.  Sync is the group's barrier.
+template <class E, int NW, class Sync>
+__device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
+    constexpr int RA = 16;  // phase A: 512 entries per warp chunk
+    constexpr int RB = 8;   // phase B: 256 outputs per warp per round
+    static_assert(NW * 32 * RB >= 2048, "phase B: one chunk of 256 outputs per warp");
+    const int K = 1 << L;
+    // Phase A -- local sort of each 512-entry chunk into K-runs (registers + shuffles).
+#pragma unroll 1
+    for (int base = w * 32 * RA; base < P; base += NW * 32 * RA) {
+        E x[RA];
+        const int e = base + lane * RA;
+#pragma unroll
+        for (int r = 0; r < RA; r += 2) {
+            if (e + r < P) {
+                b.ld2(e + r, x[r], x[r + 1]);
+            } else {
+                x[r] = E::sentinel();
+                x[r + 1] = E::sentinel();
+            }
+        }
+        wsort_runs<E, RA>(x, lane, static_cast<uint32_t>(e), L);
+#pragma unroll
+        for (int r = 0; r < RA; r += 2)
+            if (e + r < P) b.st2(e + r, x[r], x[r + 1]);
+    }
+    Sync::sync();
+    // Phase B -- rounds of merge (keep the better of paired elements of adjacent
+    // opposite runs) + rebuild (Alg. 4) until K remain.
+#pragma unroll 1
+    while (P > K) {
+        const int half = P >> 1;
+        const int obase = w * 32 * RB;
+        const int o0 = obase + lane * RB;
+        E x[RB];
+        const bool act = obase < half;
+        if (act) {
+#pragma unroll
+            for (int r = 0; r < RB; r += 2) {
+                x[r] = E::sentinel();
+                x[r + 1] = E::sentinel();
+                const int o = o0 + r;
+                if (o < half) {
+                    if (K == 1) {  // pairs (2o, 2o+1) and (2o+2, 2o+3)
+                        E a, c;
+                        b.ld2(2 * o, a, c);
+                        x[r] = esel(better(a, c), a, c);
+                        b.ld2(2 * o + 2, a, c);
+                        x[r + 1] = esel(better(a, c), a, c);
+                    } else {  // o, o+1 in one run: inputs i, i+1 and i+K, i+K+1
+                        const int i = (o << 1) - (o & (K - 1));
+                        E a0, a1, c0, c1;
+                        b.ld2(i, a0, a1);
+                        b.ld2(i + K, c0, c1);
+                        x[r] = esel(better(a0, c0), a0, c0);
+                        x[r + 1] = esel(better(a1, c1), a1, c1);
+                    }
+                }
+            }
+        }
+        Sync::sync();
+        if (act) {
+            wrebuild<E, RB>(x, lane, static_cast<uint32_t>(o0), L);
+#pragma unroll
+            for (int r = 0; r < RB; r += 2)
+                if (o0 + r < half) b.st2(o0 + r, x[r], x[r + 1]);
+        }
+        Sync::sync();
+        P = half;
+    }
+}
+
+}  // namespace topk
