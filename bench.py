@@ -1,0 +1,309 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 bitonic top-k hot path (BASELINE.json metric:
+"keys/sec and % of HBM roofline, 2^29 f32 top-k (k=1..1024), 1/2/4/8 B200").
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--k 256] [--impl ours|reference]
+
+A step is one top-k over one batch of synthetic input resident in HBM (BJ configs[1]:
+n = 2^29 uniform f32 per GPU, headline k = 256, max order, values + indices).  With
+torchrun (N > 1) every rank owns a 2^29-key shard of a global N * 2^29 input (weak
+scaling): local top-k with the shard's base offset, NCCL all-gather of the k
+candidates, one merge kernel -- the partitioned scheme of P:34 / P:444.  Rank 0 prints
+ONE JSON line.  `--impl reference` times the CPU oracle (the reference arm of this
+paper-only tier) on the host cores instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "keys/sec and % of HBM roofline, 2^29 f32 top-k (k=1..1024), 1/2/4/8 B200"
+N_PER_GPU = 1 << 29
+KEY_BYTES = 4
+FALLBACK_HBM_GBS = 6650.0  # B200_PROFILING.md fallback (only if MEASURED_PEAKS.json absent)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)", d
+    return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)", {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "20"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+            time.sleep(0.15)
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            time.sleep(0.05)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4)
+                          if len(r) > 4 + i and r[4 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons,
+                "samples": len(self.rows)}
+
+
+def dist_env():
+    r = int(os.environ.get("RANK", "0"))
+    w = int(os.environ.get("WORLD_SIZE", "1"))
+    lr = int(os.environ.get("LOCAL_RANK", "0"))
+    return r, w, lr
+
+
+def cpu_baseline(keys_host, k, note):
+    """The oracle as it stands on this host's cores (a reported baseline)."""
+    import oracle
+    t0 = time.perf_counter()
+    oracle.topk(keys_host, k, True)
+    dt = time.perf_counter() - t0
+    return {"value": keys_host.shape[0] / dt, "unit": "keys/s", "cores": oracle.threads(),
+            "kind": "oracle", "sample": note, "seconds": dt}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle timed on the host (rank 0 only)."""
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return
+    import numpy as np
+    import oracle
+    from paper_conf_sigmod_shanbhagpm18_b200 import datagen
+    oracle.build()
+    n = 1 << 26  # bounded sample: the first 2^26 rows of the 2^29-key input, every step
+    keys = datagen.generate("uniform", n, "f32", seed=datagen.config_seed(2),
+                            n_total=N_PER_GPU).numpy()
+    for _ in range(args.warmup):
+        oracle.topk(keys, args.k, True)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        oracle.topk(keys, args.k, True)
+        times.append(time.perf_counter() - t0)
+    t = sum(times)
+    value = n * args.steps / t
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "keys/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * t / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": f"2^29 uniform f32, k={args.k}, max order, values+indices (BJ configs[1])",
+                   "n": N_PER_GPU, "k": args.k, "sample_rows": n},
+        "cpu_baseline": {"value": value, "unit": "keys/s", "cores": oracle.threads(),
+                         "kind": "oracle",
+                         "sample": "first 2^26 rows of the 2^29-key input, every step"},
+        "e2e": {"value": value, "unit": "keys/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def time_steps(fn, steps, stream, torch):
+    torch.cuda.synchronize()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1)
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sigmod_shanbhagpm18_b200 as tk
+    from paper_conf_sigmod_shanbhagpm18_b200 import datagen
+
+    rank, world, lrank = dist_env()
+    if world != args.gpus:
+        args.gpus = world
+    torch.cuda.set_device(lrank)
+    dev = torch.device("cuda", lrank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    n = N_PER_GPU
+    k = args.k
+    stream = torch.cuda.current_stream(dev)
+    x = datagen.generate("uniform", n, "f32", seed=datagen.config_seed(2), device=dev,
+                         base=rank * n, n_total=world * n)
+    out_v = torch.empty(k, dtype=torch.float32, device=dev)
+    out_i = torch.empty(k, dtype=torch.int64, device=dev)
+
+    from paper_conf_sigmod_shanbhagpm18_b200.dist import sharded_topk
+
+    def step():
+        if world > 1:  # local top-k (base = shard offset) + NCCL all-gather + merge kernel
+            return sharded_topk(x, k, True, base=rank * n)
+        return tk.topk(x, k, True, base=rank * n, out=(out_v, out_i, None))
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    lc0 = tk.launch_count()
+    with ClockSampler(lrank) as clk:
+        if world > 1:
+            dist.barrier()
+        ms = time_steps(step, args.steps, stream, torch)
+    launches = tk.launch_count() - lc0
+    ms_t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms = float(ms_t.item())
+    ms_step = ms / args.steps
+    value = world * n / (ms_step / 1e3)
+
+    # ---- e2e: through the C ABI with HOST buffers (pinned); copies inside the region
+    hx = torch.empty(n, dtype=torch.float32, pin_memory=True)
+    hx.copy_(x)
+    hv = torch.empty(k, dtype=torch.float32, pin_memory=True)
+    hi = torch.empty(k, dtype=torch.int64, pin_memory=True)
+    xd = torch.empty_like(x)
+    e2e_steps = max(2, min(args.steps, 5))
+
+    def e2e_step():
+        xd.copy_(hx, non_blocking=True)
+        if world > 1:
+            v, i = sharded_topk(xd, k, True, base=rank * n)
+        else:
+            v, i = tk.topk(xd, k, True, base=rank * n, out=(out_v, out_i, None))
+        hv.copy_(v, non_blocking=True)
+        hi.copy_(i, non_blocking=True)
+
+    e2e_step()
+    ms_e2e = time_steps(e2e_step, e2e_steps, stream, torch)
+    t_e = torch.tensor([ms_e2e], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t_e, op=dist.ReduceOp.MAX)
+    e2e_value = world * n / (float(t_e.item()) / e2e_steps / 1e3)
+    del hx, xd
+
+    # ---- extra (untimed for the headline): k sweep and distributions on rank 0
+    extra = {}
+    if rank == 0 and not args.no_sweep:
+        sweep = []
+        for kk in (1, 8, 32, 64, 128, 256, 512, 1024):
+            f = lambda: tk.topk(x, kk, True)
+            for _ in range(3):
+                f()
+            t = time_steps(f, 10, stream, torch) / 10
+            sweep.append({"k": kk, "us": round(t * 1e3, 1), "keys_per_s": n / (t / 1e3)})
+        extra["k_sweep_uniform"] = sweep
+        adv = []
+        for d in ("increasing", "decreasing", "fewdistinct", "bucketkiller"):
+            xa = datagen.generate(d, n, "f32", seed=datagen.config_seed(3), device=dev)
+            f = lambda: tk.topk(xa, 256, True)
+            for _ in range(3):
+                f()
+            t = time_steps(f, 10, stream, torch) / 10
+            adv.append({"dist": d, "k": 256, "us": round(t * 1e3, 1), "keys_per_s": n / (t / 1e3)})
+            del xa
+        extra["adversarial_k256"] = adv
+
+    if rank == 0:
+        hbm, peak_src, mp = peaks()
+        gbs = n * KEY_BYTES / (ms_step / 1e3) / 1e9  # this GPU's kernel (+ merge if N > 1)
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        if os.path.exists(tp):
+            with open(tp) as f:
+                traffic = json.load(f).get(f"select_k{k}")
+        base_note = "inputs larger than L2 (2 GiB per GPU > 126 MB), no flush needed"
+        keys_host = x.cpu().numpy() if not args.no_cpu_baseline else None
+        line = {
+            "metric": METRIC, "value": value, "unit": "keys/s", "n_gpus": world,
+            "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": ms_step,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"2^29 uniform f32 per GPU, k={k}, max order, values+indices "
+                                   f"(BJ configs[1]; N>1: configs[4]-style shards + NCCL gather + merge)",
+                       "n_per_gpu": n, "n_total": world * n, "k": k,
+                       "parallelism": f"shard{world}" if world > 1 else "single",
+                       "l2": base_note},
+            "roofline": {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s",
+                         "frac": gbs / hbm, "traffic": traffic, "peak_source": peak_src,
+                         "frac_of_8tbs_nominal": gbs / 8000.0},
+            "clocks": clk.summary(),
+            "gpu_launches": launches,
+            "e2e": {"value": e2e_value, "unit": "keys/s", "h2d_bytes_per_step": n * KEY_BYTES,
+                    "d2h_bytes_per_step": k * (KEY_BYTES + 8),
+                    "note": "pinned host keys -> device copy + top-k + result copy, per step"},
+        }
+        if keys_host is not None:
+            line["cpu_baseline"] = cpu_baseline(keys_host, k, "the full 2^29-key input, once")
+        line.update(extra)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--k", type=int, default=256)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()
