@@ -114,6 +114,22 @@ topk_status_t topk_f64_kv(const double* keys, const uint32_t* payload, uint64_t 
                           uint32_t* out_payload, int64_t* out_idx, void* ws,
                           size_t ws_bytes, void* stream);
 
+/* Top-k of keys in HOST memory (pinned memory strongly recommended): the input is
+ * streamed to the device in chunks of `chunk_keys` keys through a double-buffered
+ * staging area inside `ws`; each chunk's top-k runs as soon as it has landed, so the
+ * copies overlap the reductive pass -- "the reductive nature of top-k queries makes it
+ * trivial to process the data in memory-size chunks and overlap computation with
+ * transfer" -- and the chunk results are merged (topk_merge).  h_out_keys /
+ * h_out_idx are HOST pointers, written when `stream` reaches the end of the call.
+ *   chunk_keys  multiple of 4, >= 4096; ceil(n / chunk_keys) * k <= 65536.
+ *   ws          DEVICE workspace of topk_host_workspace_bytes(dtype, n, k, chunk_keys).
+ * Uses one library-owned copy stream per device (not re-entrant across host threads). */
+size_t topk_host_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k,
+                                 uint64_t chunk_keys);
+topk_status_t topk_select_host(topk_dtype_t dtype, const void* h_keys, uint64_t n, uint32_t k,
+                               topk_order_t order, void* h_out_keys, int64_t* h_out_idx,
+                               uint64_t chunk_keys, void* ws, size_t ws_bytes, void* stream);
+
 /* Global step of the partitioned top-k (§1, App. C; multi-GPU §8(e)):
  * the exact top-k of `runs` candidate lists of `run_len` entries each, laid out
  * back to back: cand_keys[runs*run_len] (key type), cand_idx[runs*run_len] int64

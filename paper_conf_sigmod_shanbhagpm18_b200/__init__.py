@@ -16,7 +16,7 @@ import torch
 
 from . import _lib
 
-__all__ = ["topk", "merge", "Workspace", "launch_count", "workspace_bytes"]
+__all__ = ["topk", "topk_host", "merge", "Workspace", "launch_count", "workspace_bytes"]
 
 _DT = {torch.float32: _lib.F32, torch.uint32: _lib.U32, torch.float64: _lib.F64}
 
@@ -99,6 +99,40 @@ def topk(x: torch.Tensor, k: int, largest: bool = True, payload: torch.Tensor | 
                          _stream_ptr(x.device))
     _lib.check(st, "topk_select")
     return (vals, idx) if payload is None else (vals, idx, pay)
+
+
+def topk_host(x: torch.Tensor, k: int, largest: bool = True, chunk_keys: int = 1 << 26,
+              device=None, out=None):
+    """Exact top-k of a 1-D HOST tensor (pinned recommended), streamed to the GPU in
+    chunks that overlap the reductive pass.  Returns host tensors
+    ``(values, indices)``; they are valid after the current stream synchronises."""
+    if x.is_cuda or x.dim() != 1:
+        raise ValueError("topk_host expects a 1-D host tensor")
+    lib = _lib.load()
+    dt = _dtype_code(x)
+    dev = torch.device("cuda", torch.cuda.current_device()) if device is None else device
+    n = x.shape[0]
+    chunk_keys = max(4096, min(int(chunk_keys), n + (-n) % 4))
+    chunk_keys += (-chunk_keys) % 4
+    need = int(lib.topk_host_workspace_bytes(dt, n, k, chunk_keys))
+    if need == 0:
+        raise _lib.TopkError(f"invalid arguments for topk_host (n={n}, k={k})")
+    key = ("host", dev.index, need)
+    ws = _ws_cache.get(key)
+    if ws is None:
+        ws = Workspace(need, dev)
+        _ws_cache[key] = ws
+    if out is None:
+        vals = torch.empty(k, dtype=x.dtype, pin_memory=True)
+        idx = torch.empty(k, dtype=torch.int64, pin_memory=True)
+    else:
+        vals, idx = out
+    x = x.contiguous()
+    st = lib.topk_select_host(dt, _ptr(x), n, k, _lib.LARGEST if largest else _lib.SMALLEST,
+                              _ptr(vals), _ptr(idx), chunk_keys, ws.ptr(), ws.nbytes,
+                              _stream_ptr(dev))
+    _lib.check(st, "topk_select_host")
+    return vals, idx
 
 
 def merge(cand_keys: torch.Tensor, cand_idx: torch.Tensor, k: int, largest: bool = True,

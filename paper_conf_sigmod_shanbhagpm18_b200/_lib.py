@@ -23,6 +23,7 @@ SYMBOLS = (
     "topk_workspace_bytes", "topk_workspace_init", "topk_select", "topk_f32", "topk_u32",
     "topk_f64", "topk_u32_kv", "topk_f64_kv", "topk_merge_workspace_bytes", "topk_merge",
     "topk_launch_count", "topk_status_string", "topk_abi_version", "topk_probe_read",
+    "topk_host_workspace_bytes", "topk_select_host",
 )
 
 _lib = None
@@ -65,6 +66,10 @@ def load(build_if_missing: bool = True):
     lib.topk_merge.restype = i32
     lib.topk_probe_read.argtypes = [vp, sz, i32, i32, i32, i32, vp, vp]
     lib.topk_probe_read.restype = i32
+    lib.topk_host_workspace_bytes.argtypes = [i32, u64, u32, u64]
+    lib.topk_host_workspace_bytes.restype = sz
+    lib.topk_select_host.argtypes = [i32, vp, u64, u32, i32, vp, vp, u64, vp, sz, vp]
+    lib.topk_select_host.restype = i32
     lib.topk_launch_count.argtypes = []
     lib.topk_launch_count.restype = u64
     lib.topk_status_string.argtypes = [i32]

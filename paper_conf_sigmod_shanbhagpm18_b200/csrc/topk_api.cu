@@ -119,7 +119,43 @@ uint32_t tile_keys_for(topk_dtype_t dt) {
     }
 }
 
+size_t select_ws_bytes(topk_dtype_t dtype, uint32_t k, int sms) {
+    return align_up(topk::ws_cand_offset(static_cast<uint32_t>(sms)) +
+                        static_cast<size_t>(sms) * k * entry_bytes(dtype),
+                    256);
+}
+
 }  // namespace
+
+// Merge `total` candidate entries (contiguous) to the exact top-k (topk_merge's body).
+static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
+                                 const int64_t* cand_idx, const uint32_t* cand_payload,
+                                 uint64_t total, uint32_t k, topk_order_t order, void* out_keys,
+                                 uint32_t* out_payload, int64_t* out_idx, void* stream);
+// chunked-input helpers (used by topk_workspace_bytes / topk_select).  Chunk length
+// 2^31 keys; TOPK_CHUNK_N (multiple of 4) overrides it so tests can exercise the
+// chunked path on small inputs.
+static uint64_t chunk_n() {
+    static const uint64_t v = [] {
+        const char* e = std::getenv("TOPK_CHUNK_N");
+        const unsigned long long x = e ? std::strtoull(e, nullptr, 10) : 0ull;
+        return (x >= 4096 && x % 4 == 0 && x <= (1ull << 31)) ? static_cast<uint64_t>(x)
+                                                              : (1ull << 31);
+    }();
+    return v;
+}
+struct ChunkLayout {
+    size_t sel, ck, ci, cp, total;  // offsets of: select ws, cand keys, ids, payloads
+};
+static ChunkLayout chunk_layout(topk_dtype_t dtype, uint64_t nchunks, uint32_t k, int sms) {
+    ChunkLayout L;
+    L.sel = 0;
+    L.ck = align_up(select_ws_bytes(dtype, k, sms), 256);
+    L.ci = L.ck + align_up(nchunks * k * key_size(dtype), 256);
+    L.cp = L.ci + align_up(nchunks * k * 8, 256);
+    L.total = L.cp + align_up(nchunks * k * 4, 256);
+    return L;
+}
 
 extern "C" {
 
@@ -127,9 +163,9 @@ size_t topk_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k) {
     if (!valid_dtype(dtype) || n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return 0;
     int sms = 0, major = 0;
     if (!device_info(&sms, &major)) return 0;
-    return align_up(topk::ws_cand_offset(static_cast<uint32_t>(sms)) +
-                        static_cast<size_t>(sms) * k * entry_bytes(dtype),
-                    256);
+    if (n <= kMaxLaunchN && n <= chunk_n()) return select_ws_bytes(dtype, k, sms);
+    const uint64_t nch = (n + chunk_n() - 1) / chunk_n();
+    return chunk_layout(dtype, nch, k, sms).total;
 }
 
 topk_status_t topk_workspace_init(void* ws, size_t ws_bytes, void* stream) {
@@ -139,7 +175,7 @@ topk_status_t topk_workspace_init(void* ws, size_t ws_bytes, void* stream) {
     return TOPK_OK;
 }
 
-topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
+static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
                           uint64_t n, uint64_t base, uint32_t k, topk_order_t order,
                           topk_mode_t mode, void* out_keys, uint32_t* out_payload,
                           int64_t* out_idx, void* ws, size_t ws_bytes, void* stream) {
@@ -150,11 +186,10 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
     const size_t ks = key_size(dtype);
     const uintptr_t addr = reinterpret_cast<uintptr_t>(keys);
     if (addr % ks) return TOPK_ERR_INVALID_ARG;
-    if (n > kMaxLaunchN) return TOPK_ERR_UNSUPPORTED;  // chunked path: see DESIGN.md §9
     int sms = 0, major = 0;
     if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
     if (major != 10 || sms > topk::kGMax) return TOPK_ERR_UNSUPPORTED;
-    const size_t need = topk_workspace_bytes(dtype, n, k);
+    const size_t need = select_ws_bytes(dtype, k, sms);
     if (!ws || ws_bytes < need || (reinterpret_cast<uintptr_t>(ws) % 256)) return TOPK_ERR_WORKSPACE;
 
     topk::SelectParams p;
@@ -219,6 +254,44 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
     return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
 }
 
+
+// Inputs longer than one launch indexes (32-bit local row ids): chunks of chunk_n() keys,
+// each reduced by its own launch with its base offset (global ids), then the merge
+// kernel -- the decomposition the paper uses across cores.
+
+topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
+                          uint64_t n, uint64_t base, uint32_t k, topk_order_t order,
+                          topk_mode_t mode, void* out_keys, uint32_t* out_payload,
+                          int64_t* out_idx, void* ws, size_t ws_bytes, void* stream) {
+    if (n <= kMaxLaunchN && n <= chunk_n())
+        return select_one(dtype, keys, payload, n, base, k, order, mode, out_keys, out_payload,
+                          out_idx, ws, ws_bytes, stream);
+    if (!valid_dtype(dtype) || !keys || k == 0 || k > TOPK_MAX_K) return TOPK_ERR_INVALID_ARG;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    const uint64_t nch = (n + chunk_n() - 1) / chunk_n();
+    if (nch * k > 65536) return TOPK_ERR_UNSUPPORTED;
+    const ChunkLayout L = chunk_layout(dtype, nch, k, sms);
+    if (!ws || ws_bytes < L.total) return TOPK_ERR_WORKSPACE;
+    unsigned char* w = static_cast<unsigned char*>(ws);
+    const size_t ks = key_size(dtype);
+    uint64_t total = 0;
+    for (uint64_t c = 0; c < nch; ++c) {
+        const uint64_t lo = c * chunk_n(), len = (n - lo < chunk_n()) ? n - lo : chunk_n();
+        const uint32_t kc = len < k ? static_cast<uint32_t>(len) : k;  // ragged last chunk
+        topk_status_t st = select_one(
+            dtype, static_cast<const unsigned char*>(keys) + lo * ks,
+            payload ? payload + lo : nullptr, len, base + lo, kc, order, mode,
+            w + L.ck + total * ks, payload ? reinterpret_cast<uint32_t*>(w + L.cp) + total : nullptr,
+            reinterpret_cast<int64_t*>(w + L.ci) + total, w + L.sel, L.ck, stream);
+        if (st != TOPK_OK) return st;
+        total += kc;
+    }
+    return merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
+                       payload ? reinterpret_cast<const uint32_t*>(w + L.cp) : nullptr, total, k,
+                       order, out_keys, out_payload, out_idx, stream);
+}
+
 topk_status_t topk_f32(const float* keys, uint64_t n, uint32_t k, topk_order_t order,
                        float* out_keys, int64_t* out_idx, void* ws, size_t ws_bytes,
                        void* stream) {
@@ -268,33 +341,10 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
                          size_t ws_bytes, void* stream) {
     (void)ws;
     (void)ws_bytes;
-    if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
-    if (!cand_keys || !cand_idx || runs == 0 || run_len == 0) return TOPK_ERR_INVALID_ARG;
-    const uint64_t total = static_cast<uint64_t>(runs) * run_len;
-    if (total > 65536 || k == 0 || k > TOPK_MAX_K || k > total) return TOPK_ERR_INVALID_ARG;
-    if (out_payload && !cand_payload) return TOPK_ERR_INVALID_ARG;
-    int sms = 0, major = 0;
-    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
-    if (major != 10) return TOPK_ERR_UNSUPPORTED;
-    topk::MergeParams p;
-    p.cand_keys = cand_keys;
-    p.cand_idx = cand_idx;
-    p.cand_payload = cand_payload;
-    p.out_keys = out_keys;
-    p.out_payload = out_payload;
-    p.out_idx = out_idx;
-    p.total = static_cast<uint32_t>(total);
-    p.k = k;
-    p.K = next_pow2_u32(k);
-    cudaStream_t st = static_cast<cudaStream_t>(stream);
-    const bool mn = order == TOPK_SMALLEST;
-    cudaError_t e;
-    switch (dtype) {
-        case TOPK_F32: e = dispatch_merge<float>(p, mn, st); break;
-        case TOPK_U32: e = dispatch_merge<uint32_t>(p, mn, st); break;
-        default: e = dispatch_merge<double>(p, mn, st); break;
-    }
-    return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+    if (runs == 0 || run_len == 0) return TOPK_ERR_INVALID_ARG;
+    return merge_total(dtype, cand_keys, cand_idx, cand_payload,
+                       static_cast<uint64_t>(runs) * run_len, k, order, out_keys, out_payload,
+                       out_idx, stream);
 }
 
 /* Debug (not in topk.h's stable surface): read / reset the device counters of
@@ -368,6 +418,103 @@ int topk_debug_trace(int enable, uint64_t* host) {
     return 0;
 }
 
+// ---- host-resident input: chunked H2D overlapped with the reductive pass ----
+struct HostLayout {
+    size_t stage[2], ck, ci, sel, ok, oi, total;
+};
+static HostLayout host_layout(topk_dtype_t dtype, uint64_t n, uint32_t k, uint64_t chunk,
+                              int sms) {
+    const size_t ks = key_size(dtype);
+    const uint64_t nch = (n + chunk - 1) / chunk;
+    HostLayout L;
+    L.stage[0] = 0;
+    L.stage[1] = align_up(chunk * ks, 256);
+    L.ck = L.stage[1] + align_up(chunk * ks, 256);
+    L.ci = L.ck + align_up(nch * k * ks, 256);
+    L.sel = L.ci + align_up(nch * k * 8, 256);
+    L.ok = L.sel + align_up(select_ws_bytes(dtype, k, sms), 256);
+    L.oi = L.ok + align_up(k * ks, 256);
+    L.total = L.oi + align_up(k * 8, 256);
+    return L;
+}
+
+size_t topk_host_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k,
+                                 uint64_t chunk_keys) {
+    if (!valid_dtype(dtype) || n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return 0;
+    if (chunk_keys < 4096 || (chunk_keys % 4) || chunk_keys > kMaxLaunchN) return 0;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return 0;
+    return host_layout(dtype, n, k, chunk_keys, sms).total;
+}
+
+topk_status_t topk_select_host(topk_dtype_t dtype, const void* h_keys, uint64_t n, uint32_t k,
+                               topk_order_t order, void* h_out_keys, int64_t* h_out_idx,
+                               uint64_t chunk_keys, void* ws, size_t ws_bytes, void* stream) {
+    if (!valid_dtype(dtype) || !valid_order(order) || !h_keys) return TOPK_ERR_INVALID_ARG;
+    if (n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return TOPK_ERR_INVALID_ARG;
+    if (chunk_keys < 4096 || (chunk_keys % 4) || chunk_keys > kMaxLaunchN)
+        return TOPK_ERR_INVALID_ARG;
+    const uint64_t nch = (n + chunk_keys - 1) / chunk_keys;
+    if (nch * k > 65536) return TOPK_ERR_INVALID_ARG;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    const HostLayout L = host_layout(dtype, n, k, chunk_keys, sms);
+    if (!ws || ws_bytes < L.total || (reinterpret_cast<uintptr_t>(ws) % 256))
+        return TOPK_ERR_WORKSPACE;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev >= 64) return TOPK_ERR_CUDA;
+    // library-owned copy stream + events, one set per device
+    static cudaStream_t copy_st[64];
+    static cudaEvent_t copied[64][2], freed[64][2], start[64];
+    if (!copy_st[dev]) {
+        if (cudaStreamCreateWithFlags(&copy_st[dev], cudaStreamNonBlocking) != cudaSuccess)
+            return TOPK_ERR_CUDA;
+        for (int b = 0; b < 2; ++b) {
+            cudaEventCreateWithFlags(&copied[dev][b], cudaEventDisableTiming);
+            cudaEventCreateWithFlags(&freed[dev][b], cudaEventDisableTiming);
+        }
+        cudaEventCreateWithFlags(&start[dev], cudaEventDisableTiming);
+    }
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    cudaStream_t cp = copy_st[dev];
+    unsigned char* w = static_cast<unsigned char*>(ws);
+    const size_t ks = key_size(dtype);
+    // the staging buffers may still be read by earlier work on `stream`
+    if (cudaEventRecord(start[dev], st) != cudaSuccess) return TOPK_ERR_CUDA;
+    cudaStreamWaitEvent(cp, start[dev], 0);
+    uint64_t total = 0;
+    for (uint64_t c = 0; c < nch; ++c) {
+        const int b = static_cast<int>(c & 1);
+        const uint64_t lo = c * chunk_keys;
+        const uint64_t len = (n - lo < chunk_keys) ? n - lo : chunk_keys;
+        if (c >= 2) cudaStreamWaitEvent(cp, freed[dev][b], 0);
+        if (cudaMemcpyAsync(w + L.stage[b], static_cast<const unsigned char*>(h_keys) + lo * ks,
+                            len * ks, cudaMemcpyHostToDevice, cp) != cudaSuccess)
+            return TOPK_ERR_CUDA;
+        cudaEventRecord(copied[dev][b], cp);
+        cudaStreamWaitEvent(st, copied[dev][b], 0);
+        const uint32_t kc = len < k ? static_cast<uint32_t>(len) : k;  // ragged last chunk
+        topk_status_t r = select_one(dtype, w + L.stage[b], nullptr, len, lo, kc, order,
+                                     TOPK_MODE_FILTER, w + L.ck + total * ks, nullptr,
+                                     reinterpret_cast<int64_t*>(w + L.ci) + total, w + L.sel,
+                                     L.ok - L.sel, stream);
+        if (r != TOPK_OK) return r;
+        cudaEventRecord(freed[dev][b], st);
+        total += kc;
+    }
+    topk_status_t r = merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
+                                  nullptr, total, k, order, w + L.ok, nullptr,
+                                  reinterpret_cast<int64_t*>(w + L.oi), stream);
+    if (r != TOPK_OK) return r;
+    if (h_out_keys &&
+        cudaMemcpyAsync(h_out_keys, w + L.ok, k * ks, cudaMemcpyDeviceToHost, st) != cudaSuccess)
+        return TOPK_ERR_CUDA;
+    if (h_out_idx &&
+        cudaMemcpyAsync(h_out_idx, w + L.oi, k * 8, cudaMemcpyDeviceToHost, st) != cudaSuccess)
+        return TOPK_ERR_CUDA;
+    return cudaGetLastError() == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+}
+
 uint64_t topk_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
 
 const char* topk_status_string(topk_status_t s) {
@@ -384,3 +531,35 @@ const char* topk_status_string(topk_status_t s) {
 int topk_abi_version(void) { return TOPK_ABI_VERSION; }
 
 }  // extern "C"
+
+static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
+                                 const int64_t* cand_idx, const uint32_t* cand_payload,
+                                 uint64_t total, uint32_t k, topk_order_t order, void* out_keys,
+                                 uint32_t* out_payload, int64_t* out_idx, void* stream) {
+    if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
+    if (!cand_keys || !cand_idx || total == 0) return TOPK_ERR_INVALID_ARG;
+    if (total > 65536 || k == 0 || k > TOPK_MAX_K || k > total) return TOPK_ERR_INVALID_ARG;
+    if (out_payload && !cand_payload) return TOPK_ERR_INVALID_ARG;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    if (major != 10) return TOPK_ERR_UNSUPPORTED;
+    topk::MergeParams p;
+    p.cand_keys = cand_keys;
+    p.cand_idx = cand_idx;
+    p.cand_payload = cand_payload;
+    p.out_keys = out_keys;
+    p.out_payload = out_payload;
+    p.out_idx = out_idx;
+    p.total = static_cast<uint32_t>(total);
+    p.k = k;
+    p.K = next_pow2_u32(k);
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const bool mn = order == TOPK_SMALLEST;
+    cudaError_t e;
+    switch (dtype) {
+        case TOPK_F32: e = dispatch_merge<float>(p, mn, st); break;
+        case TOPK_U32: e = dispatch_merge<uint32_t>(p, mn, st); break;
+        default: e = dispatch_merge<double>(p, mn, st); break;
+    }
+    return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+}
