@@ -331,38 +331,43 @@ struct Ctx {
     unsigned long long* scratch;  // shared [J][G]
     int k, K;
     int G, gmax, J;
+    int j_lo, nrows;  // rank-bound rows used: j_lo .. j_lo + nrows - 1 (t <= G)
     bool filter;
 };
 
-// Rank bound over scratch[J][G] (0 = missing sample): for row j the t-th largest word,
-// t = ceil(k / 2^j) <= G.  Collective (consumers); st->best[] receives one word per
-// row.  Entry: scratch filled and barrier passed; exit: after a barrier.
+// Rank bound over scratch[nrows][G] (row r = sample row j_lo + r; 0 = missing sample):
+// the t-th largest word of row j, t = ceil(k / 2^j) <= G.  Only the nrows (<= 3) rows
+// with the smallest valid j are ranked -- they give the tightest bounds (a deeper row
+// samples a weaker quantile of every run).  Collective (consumers); st->best[] gets one
+// word per row.  Entry: scratch filled and barrier passed; exit: after a barrier.
 template <class E, class Key>
 __device__ void rank_rows(CtaState<E, Key>* st, const Ctx& cx) {
     if (threadIdx.x < kPubRows) st->best[threadIdx.x] = 0ull;
     CSync::sync();
-    const int JG = cx.J * cx.G;
-    for (int q = threadIdx.x; q < JG; q += kNC) {
-        const int ji = q / cx.G;
+    const int RG = cx.nrows * cx.G;
+    for (int q = threadIdx.x; q < RG; q += kNC) {
+        const int r = q / cx.G;
+        const int ji = cx.j_lo + r;
         const int t = (cx.k + (1 << ji) - 1) >> ji;
         const unsigned long long v = cx.scratch[q];
-        if (t > cx.G || v == 0ull) continue;
-        const unsigned long long* row = cx.scratch + ji * cx.G;
+        if (v == 0ull) continue;
+        const unsigned long long* row = cx.scratch + r * cx.G;
         int rank = 0;
+#pragma unroll 4
         for (int c2 = 0; c2 < cx.G; ++c2) rank += row[c2] > v ? 1 : 0;
         if (rank == t - 1) st->best[ji] = v;  // unique: samples are distinct entries
     }
     CSync::sync();
 }
 
-// Load every CTA's published samples into shared scratch (stale values are smaller,
-// still valid).
+// Load every CTA's published samples of the ranked rows into shared scratch (stale
+// values are smaller, still valid).
 __device__ __forceinline__ void load_pub(const Ctx& cx) {
-    const int JG = cx.J * cx.G;
-    for (int q = threadIdx.x; q < JG; q += kNC) {
-        const int ji = q / cx.G, cc = q % cx.G;
-        cx.scratch[q] = ld_relaxed_u64(
-            reinterpret_cast<const uint64_t*>(cx.pub + static_cast<size_t>(ji) * cx.gmax + cc));
+    const int RG = cx.nrows * cx.G;
+    for (int q = threadIdx.x; q < RG; q += kNC) {
+        const int r = q / cx.G, cc = q % cx.G;
+        cx.scratch[q] = ld_relaxed_u64(reinterpret_cast<const uint64_t*>(
+            cx.pub + static_cast<size_t>(cx.j_lo + r) * cx.gmax + cc));
     }
 }
 
@@ -404,10 +409,7 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
     for (int i = K + cnt + threadIdx.x; i < P; i += kNC) buf.st(i, E::sentinel());
     CSync::sync();
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (K <= 256)
-        wnet_topk<E, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
-    else
-        bitonic_topk_smem<E, kNC, CSync>(buf, P, K);
+    wnet_topk<E, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
     const E kth = buf.ld(k - 1);
     const bool publish = mode == kFlushStream && cx.filter;
     const bool ranks = publish && st->nflush > 0;
@@ -597,6 +599,9 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     cx.G = static_cast<int>(G);
     cx.gmax = static_cast<int>(p.gmax);
     cx.J = static_cast<int>(p.J);
+    cx.j_lo = 0;
+    while (cx.j_lo < cx.J && ((k + (1 << cx.j_lo) - 1) >> cx.j_lo) > cx.G) ++cx.j_lo;
+    cx.nrows = cx.J - cx.j_lo < 3 ? cx.J - cx.j_lo : 3;
     cx.filter = FILTER;
 
     for (int i = tid; i < K; i += kNT) buf.st(i, E::sentinel());
@@ -747,12 +752,14 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // (1) Rank bound over the final runs (tail form of the flush bound): row j holds
         // each run's 2^j-th best; the t-th largest (t = ceil(k / 2^j) <= G) bounds the
         // global k-th best.  All loads in one parallel pass.
-        for (int q = tid; q < cx.J * cx.G; q += kNC) {
-            const int ji = q / cx.G, cc = q % cx.G;
+        for (int q = tid; q < cx.nrows * cx.G; q += kNC) {
+            const int ji = cx.j_lo + q / cx.G, cc = q % cx.G;
             scratch[q] = bound_word(cand.ld(static_cast<size_t>(cc) * k + (1u << ji) - 1u));
         }
         CSync::sync();
+        if (tid == 0) trace(8);
         rank_rows(&st, cx);
+        if (tid == 0) trace(9);
         if (tid == 0) {
             E tb = from_bound_word<E>(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&hdr->tau_g)));
             for (int ji = 0; ji < cx.J; ++ji) {
@@ -772,11 +779,23 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         for (int q = tid; q < (kGMax + 31) / 32; q += kNC) s_more[q] = 0u;
         CSync::sync();
         constexpr int CI = 8;
+        __shared__ int s_flag_list[kGMax];
+        __shared__ int s_nflag;
         for (int phase = 0; phase < 2; ++phase) {
+            if (phase == 1) {  // compact the runs whose 32nd entry still qualified
+                if (tid == 0) {
+                    int nf = 0;
+                    for (int cc = 0; cc < cx.G; ++cc)
+                        if ((s_more[cc >> 5] >> (cc & 31)) & 1u) s_flag_list[nf++] = cc;
+                    s_nflag = nf;
+                }
+                CSync::sync();
+            }
             const int lo = phase == 0 ? 0 : kk;
             const int span = phase == 0 ? kk : k - kk;
-            if (span <= 0) break;
-            const int total = cx.G * span;
+            const int nruns = phase == 0 ? cx.G : s_nflag;
+            if (span <= 0 || nruns == 0) break;
+            const int total = nruns * span;
             for (int q0 = 0; q0 < total; q0 += CI * kNC) {
                 E ents[CI];
                 uint32_t mask = 0;
@@ -785,9 +804,9 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                     const int q = q0 + tid + r * kNC;
                     ents[r] = E::sentinel();
                     if (q >= total) continue;
-                    const int cc = q / span, j = lo + q % span;
+                    const int cc = phase == 0 ? q / span : s_flag_list[q / span];
+                    const int j = lo + q % span;
                     if (cc == static_cast<int>(c)) continue;
-                    if (phase == 1 && !((s_more[cc >> 5] >> (cc & 31)) & 1u)) continue;
                     const E e = cand.ld(static_cast<size_t>(cc) * k + j);
                     if (!e.is_sentinel() && !better(tb, e)) {
                         ents[r] = e;
@@ -814,6 +833,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             }
             CSync::sync();
         }
+        if (tid == 0) trace(10);
         if (st.cnt > 0) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
     }
     // ---- finalize: best first, original key bits, global index, payload ----

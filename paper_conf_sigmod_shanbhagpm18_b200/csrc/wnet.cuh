@@ -116,16 +116,12 @@ __device__ __forceinline__ void wrebuild(E (&x)[R], int lane, uint32_t e0, int L
     for (int b = L - 1; b >= 0; --b) wstep<E, R>(x, lane, e0, b, L);
 }
 
-// Bitonic top-K (K = 2^L <= 256) of b[0..P), P a power of two, 2K <= P <= 4096, by
-// the NW warps of the calling group (warp index w, lane), all of which call this.
-// Result: b[0..K) best first.  Sync is the group's barrier.
-template <class E, int NW, class Sync>
-__device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
-    constexpr int RA = 16;  // phase A: 512 entries per warp chunk
-    constexpr int RB = 8;   // phase B: 256 outputs per warp per round
-    static_assert(NW * 32 * RB >= 2048, "phase B: one chunk of 256 outputs per warp");
-    const int K = 1 << L;
-    // Phase A -- local sort of each 512-entry chunk into K-runs (registers + shuffles).
+// Register pass over 512-entry chunks of b[0..P): steps b = hi .. 0 with direction
+// bit d (all within a chunk: bits 0-3 registers, 4-8 shuffles).
+template <class E, int NW>
+__device__ __forceinline__ void wchunk_steps(const SBuf<E>& b, int P, int hi, int d, int w,
+                                             int lane) {
+    constexpr int RA = 16;
 #pragma unroll 1
     for (int base = w * 32 * RA; base < P; base += NW * 32 * RA) {
         E x[RA];
@@ -139,12 +135,97 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
                 x[r + 1] = E::sentinel();
             }
         }
-        wsort_runs<E, RA>(x, lane, static_cast<uint32_t>(e), L);
+#pragma unroll 1
+        for (int bb = hi; bb >= 0; --bb) wstep<E, RA>(x, lane, static_cast<uint32_t>(e), bb, d);
+#pragma unroll
+        for (int r = 0; r < RA; r += 2)
+            if (e + r < P) b.st2(e + r, x[r], x[r + 1]);
+    }
+}
+
+// Shared-memory step on bit bb >= 9 (pairs in different 512-chunks), Alg. 4 index math.
+template <class E, int NT, class Sync>
+__device__ __forceinline__ void wsmem_step(const SBuf<E>& b, int P, int bb, int d) {
+    const int inc = 1 << bb, dir = 1 << d;
+    for (int t = threadIdx.x; t < (P >> 1); t += NT) {
+        const int i = (t << 1) - (t & (inc - 1));
+        const int j = i + inc;
+        const bool best_first = (i & dir) == 0;
+        const E x0 = b.ld(i), x1 = b.ld(j);
+        const bool sw = best_first == better(x1, x0);
+        b.st(i, esel(sw, x1, x0));
+        b.st(j, esel(sw, x0, x1));
+    }
+    Sync::sync();
+}
+
+// Bitonic top-K (K = 2^L <= 1024) of b[0..P), P a power of two, 2K <= P <= 4096, by
+// the NW warps of the calling group (warp index w, lane), all of which call this.
+// Result: b[0..K) best first.  Sync is the group's barrier.  Steps on element bits
+// 0-8 run in registers / shuffles; the rare bit-9 steps (K = 1024) in shared memory.
+template <class E, int NW, class Sync>
+__device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
+    constexpr int RA = 16;  // phase A: 512 entries per warp chunk
+    constexpr int RB = 8;   // phase B: 256 outputs per warp per round
+    static_assert(NW * 32 * RB >= 2048, "phase B: one chunk of 256 outputs per warp");
+    const int K = 1 << L;
+    // Phase A -- local sort of each 512-entry chunk into min(K, 512)-runs (registers).
+    const int LA = L < 9 ? L : 9;
+#pragma unroll 1
+    for (int base = w * 32 * RA; base < P; base += NW * 32 * RA) {
+        E x[RA];
+        const int e = base + lane * RA;
+#pragma unroll
+        for (int r = 0; r < RA; r += 2) {
+            if (e + r < P) {
+                b.ld2(e + r, x[r], x[r + 1]);
+            } else {
+                x[r] = E::sentinel();
+                x[r + 1] = E::sentinel();
+            }
+        }
+        wsort_runs<E, RA>(x, lane, static_cast<uint32_t>(e), LA);
 #pragma unroll
         for (int r = 0; r < RA; r += 2)
             if (e + r < P) b.st2(e + r, x[r], x[r + 1]);
     }
     Sync::sync();
+    if (L == 10) {  // last local-sort stage (len 512): bit 9 in smem, bits 8..0 in registers
+        wsmem_step<E, NW * 32, Sync>(b, P, 9, 10);
+        wchunk_steps<E, NW>(b, P, 8, 10, w, lane);
+        Sync::sync();
+    }
+    if (L >= 9) {
+        // Phase B for K >= 512: merge through registers + shared memory, rebuild with
+        // the same hybrid steps.
+#pragma unroll 1
+        while (P > K) {
+            const int half = P >> 1;
+            constexpr int PER = 4096 / 2 / (NW * 32) + 1;
+            E keep[PER];
+#pragma unroll
+            for (int r = 0; r < PER; ++r) {
+                const int o = threadIdx.x + r * NW * 32;
+                if (o < half) {
+                    const int i = (o << 1) - (o & (K - 1));
+                    const E a = b.ld(i), c = b.ld(i + K);
+                    keep[r] = esel(better(a, c), a, c);
+                }
+            }
+            Sync::sync();
+#pragma unroll
+            for (int r = 0; r < PER; ++r) {
+                const int o = threadIdx.x + r * NW * 32;
+                if (o < half) b.st(o, keep[r]);
+            }
+            Sync::sync();
+            P = half;
+            if (L == 10) wsmem_step<E, NW * 32, Sync>(b, P, 9, 10);
+            wchunk_steps<E, NW>(b, P, 8, L, w, lane);
+            Sync::sync();
+        }
+        return;
+    }
     // Phase B -- rounds of merge (keep the better of paired elements of adjacent
     // opposite runs) + rebuild (Alg. 4) until K remain.
 #pragma unroll 1
