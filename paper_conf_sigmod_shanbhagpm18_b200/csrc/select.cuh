@@ -587,7 +587,12 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     const int K = static_cast<int>(p.K);
     const int k = static_cast<int>(p.k);
     // Until a bound exists, keep the buffer small so the first flush is cheap.
-    const int boot_limit = FILTER ? (K > 1024 ? K : 1024) : kCap - K;
+#ifndef TOPK_BOOT_BIG_K
+#define TOPK_BOOT_BIG_K 32
+#endif
+    // (K >= TOPK_BOOT_BIG_K: fill the whole buffer -- one larger boot flush whose run,
+    // after the rank refresh, bounds tightly enough that no second flush is needed)
+    const int boot_limit = !FILTER ? kCap - K : (K >= TOPK_BOOT_BIG_K ? kCap - K : 1024);
     const Key* keys = static_cast<const Key*>(p.keys);
     WsHeader* hdr = reinterpret_cast<WsHeader*>(p.ws);
     Ctx cx;

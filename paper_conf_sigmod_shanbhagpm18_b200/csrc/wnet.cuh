@@ -24,6 +24,9 @@
 
 namespace topk {
 
+// netbench instrumentation: clock64 at the end of phase A of the last network call
+__device__ long long g_wnet_phase_a_end;
+
 template <class E>
 __device__ __forceinline__ E shfl_xor_e(const E& e, int m);
 template <>
@@ -73,14 +76,11 @@ template <class E, int R>
 __device__ __forceinline__ void wstep(E (&x)[R], int lane, uint32_t e0, int b, int d) {
     constexpr int LR = Log2<R>::v;
     if (b < LR) {
-        uint32_t wm;
-        if (d < LR) {
-            wm = 0;
-#pragma unroll
-            for (int r = 0; r < R; ++r) wm |= ((static_cast<uint32_t>(r) >> d) & 1u) << r;
-        } else {
-            wm = ((e0 >> d) & 1u) ? 0xFFFFFFFFu : 0u;
-        }
+        // bit r of wm = bit d of register index r (d < LR), or bit d of e0 for all r:
+        // the patterns 0xAAAA, 0xCCCC, 0xF0F0, 0xFF00 for d = 0..3 packed in one word
+        const uint32_t wm =
+            d < LR ? static_cast<uint32_t>((0xFF00F0F0CCCCAAAAull >> (16 * d)) & 0xFFFFull)
+                   : (((e0 >> d) & 1u) ? 0xFFFFFFFFu : 0u);
         switch (b) {
             case 0: reg_step<E, R, 0>(x, wm); break;
             case 1: if constexpr (LR > 1) reg_step<E, R, 1>(x, wm); break;
@@ -169,27 +169,52 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
     constexpr int RB = 8;   // phase B: 256 outputs per warp per round
     static_assert(NW * 32 * RB >= 2048, "phase B: one chunk of 256 outputs per warp");
     const int K = 1 << L;
-    // Phase A -- local sort of each 512-entry chunk into min(K, 512)-runs (registers).
+    // Phase A -- local sort into min(K, 512)-runs in registers.  Small buffers use
+    // 256-entry chunks (8 per lane) so twice as many warps share the latency-bound
+    // step chain; K >= 512 or P > 2048 use 512-entry chunks (16 per lane).
     const int LA = L < 9 ? L : 9;
-#pragma unroll 1
-    for (int base = w * 32 * RA; base < P; base += NW * 32 * RA) {
-        E x[RA];
-        const int e = base + lane * RA;
+    if (L <= 8 && P <= 8 * 256 && NW >= 8) {
+        constexpr int R8 = 8;
+        const int base = w * 32 * R8;
+        if (base < P) {
+            E x[R8];
+            const int e = base + lane * R8;
 #pragma unroll
-        for (int r = 0; r < RA; r += 2) {
-            if (e + r < P) {
-                b.ld2(e + r, x[r], x[r + 1]);
-            } else {
-                x[r] = E::sentinel();
-                x[r + 1] = E::sentinel();
+            for (int r = 0; r < R8; r += 2) {
+                if (e + r < P) {
+                    b.ld2(e + r, x[r], x[r + 1]);
+                } else {
+                    x[r] = E::sentinel();
+                    x[r + 1] = E::sentinel();
+                }
             }
-        }
-        wsort_runs<E, RA>(x, lane, static_cast<uint32_t>(e), LA);
+            wsort_runs<E, R8>(x, lane, static_cast<uint32_t>(e), LA);
 #pragma unroll
-        for (int r = 0; r < RA; r += 2)
-            if (e + r < P) b.st2(e + r, x[r], x[r + 1]);
+            for (int r = 0; r < R8; r += 2)
+                if (e + r < P) b.st2(e + r, x[r], x[r + 1]);
+        }
+    } else {
+#pragma unroll 1
+        for (int base = w * 32 * RA; base < P; base += NW * 32 * RA) {
+            E x[RA];
+            const int e = base + lane * RA;
+#pragma unroll
+            for (int r = 0; r < RA; r += 2) {
+                if (e + r < P) {
+                    b.ld2(e + r, x[r], x[r + 1]);
+                } else {
+                    x[r] = E::sentinel();
+                    x[r + 1] = E::sentinel();
+                }
+            }
+            wsort_runs<E, RA>(x, lane, static_cast<uint32_t>(e), LA);
+#pragma unroll
+            for (int r = 0; r < RA; r += 2)
+                if (e + r < P) b.st2(e + r, x[r], x[r + 1]);
+        }
     }
     Sync::sync();
+    if (threadIdx.x == 0) g_wnet_phase_a_end = clock64();
     if (L == 10) {  // last local-sort stage (len 512): bit 9 in smem, bits 8..0 in registers
         wsmem_step<E, NW * 32, Sync>(b, P, 9, 10);
         wchunk_steps<E, NW>(b, P, 8, 10, w, lane);

@@ -11,4 +11,4 @@ for e64 in (0, 1):
             if P < 2 << L: continue
             for smem_net in ((0, 1) if L <= 8 else (1,)):
                 lib.topk_debug_netbench(P, L, e64, smem_net, 20, out)
-                print(json.dumps(dict(e64=e64, L=L, P=P, net="smem" if smem_net else "warp", cycles=out[0])), flush=True)
+                print(json.dumps(dict(e64=e64, L=L, P=P, net="smem" if smem_net else "warp", cycles=out[0], phaseA=out[1] if not smem_net else None)), flush=True)
