@@ -257,6 +257,48 @@ def run_ours(args):
             adv.append({"dist": d, "k": 256, "us": round(t * 1e3, 1), "keys_per_s": n / (t / 1e3)})
             del xa
         extra["adversarial_k256"] = adv
+        # the other BJ configs on this GPU (parity-tested in tests/; reported here)
+        cfgs = []
+
+        def timed(f, it=10):
+            for _ in range(3):
+                f()
+            return time_steps(f, it, stream, torch) / it
+
+        x1 = datagen.generate("uniform", 1 << 20, "f32", seed=datagen.config_seed(1), device=dev)
+        t = timed(lambda: tk.topk(x1, 32, True), 50)
+        cfgs.append({"config": "BJ1: 2^20 uniform f32, k=32 (launch-bound)", "us": round(t * 1e3, 1),
+                     "keys_per_s": (1 << 20) / (t / 1e3)})
+        del x1
+        n4 = 1 << 28
+        xu = datagen.generate("uniform", n4, "u32", seed=datagen.config_seed(4), device=dev)
+        pu = datagen.payload(n4, seed=datagen.config_seed(4), device=dev)
+        t = timed(lambda: tk.topk(xu, 64, True, payload=pu))
+        cfgs.append({"config": "BJ4a: 2^28 u32 key + u32 payload, DESC LIMIT 64", "us": round(t * 1e3, 1),
+                     "keys_per_s": n4 / (t / 1e3), "frac_hbm": n4 * 4 / (t / 1e3) / 1e9 / peaks()[0]})
+        del xu, pu
+        xd64 = datagen.generate("uniform", n4, "f64", seed=datagen.config_seed(4), device=dev)
+        t = timed(lambda: tk.topk(xd64, 64, True))
+        cfgs.append({"config": "BJ4b: 2^28 f64, DESC LIMIT 64", "us": round(t * 1e3, 1),
+                     "keys_per_s": n4 / (t / 1e3), "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
+        del xd64
+        for kk in (32, 256):
+            t = timed(lambda: tk.topk(x, kk, True, mode="pure"), 2)
+            cfgs.append({"config": f"pure mode (paper's data-independent network on every key), "
+                                   f"2^29 f32, k={kk}", "us": round(t * 1e3, 1),
+                         "keys_per_s": n / (t / 1e3)})
+        if not args.no_big:
+            del x
+            torch.cuda.empty_cache()
+            n5 = 1 << 32
+            x5 = datagen.generate("uniform", n5, "f32", seed=datagen.config_seed(5), device=dev)
+            t = timed(lambda: tk.topk(x5, 256, True), 5)
+            cfgs.append({"config": "BJ5 at G=1: 2^32 uniform f32, k=256 (2 chunks of 2^31 + merge)",
+                         "us": round(t * 1e3, 1), "keys_per_s": n5 / (t / 1e3),
+                         "frac_hbm": n5 * 4 / (t / 1e3) / 1e9 / peaks()[0]})
+            del x5
+            x = None
+        extra["other_configs"] = cfgs
 
     if rank == 0:
         hbm, peak_src, mp = peaks()
@@ -267,7 +309,10 @@ def run_ours(args):
             with open(tp) as f:
                 traffic = json.load(f).get(f"select_k{k}")
         base_note = "inputs larger than L2 (2 GiB per GPU > 126 MB), no flush needed"
-        keys_host = x.cpu().numpy() if not args.no_cpu_baseline else None
+        keys_host = None
+        if not args.no_cpu_baseline:
+            keys_host = datagen.generate("uniform", n, "f32", seed=datagen.config_seed(2),
+                                         base=0, n_total=world * n).numpy()
         line = {
             "metric": METRIC, "value": value, "unit": "keys/s", "n_gpus": world,
             "steps": args.steps, "warmup": max(3, args.warmup), "ms_per_step": ms_step,
@@ -307,6 +352,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-big", action="store_true", help="skip the 2^32-key extra")
     args = ap.parse_args()
     if args.impl == "reference":
         run_reference(args)

@@ -311,9 +311,9 @@ __device__ unsigned long long g_stats[8];
 // 5 tail begin, 6 end, 7 refresh); g_trace[c][0] = count.  Enabled by g_trace_on.
 constexpr int kTraceCtas = 160, kTraceLen = 64;
 __device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
-__device__ int g_trace_on;
+__device__ __constant__ int c_trace_on;  // set by topk_debug_trace (constant bank: free)
 __device__ __forceinline__ void trace(int ev) {
-    if (!g_trace_on || blockIdx.x >= kTraceCtas) return;
+    if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     unsigned long long* row = g_trace[blockIdx.x];
@@ -776,6 +776,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         }
         CSync::sync();
         const E tb = st.tau;
+        if (tid == 0) trace(11);
         // (2) Every run is sorted best first, so only a prefix can be >= tb: append the
         // qualifying entries of the first min(k, 32) of every other run (one parallel
         // pass), then the rest of the runs whose 32nd entry still qualified (rare).
@@ -783,16 +784,23 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         __shared__ unsigned int s_more[(kGMax + 31) / 32];
         for (int q = tid; q < (kGMax + 31) / 32; q += kNC) s_more[q] = 0u;
         CSync::sync();
-        constexpr int CI = 8;
+        constexpr int CI = 11;  // one pass covers G * 32 <= 160 * 32 = 5120 <= 11 * 480
         __shared__ int s_flag_list[kGMax];
         __shared__ int s_nflag;
         for (int phase = 0; phase < 2; ++phase) {
+            if (tid == 0) trace(12 + phase);
             if (phase == 1) {  // compact the runs whose 32nd entry still qualified
-                if (tid == 0) {
+                if (kk >= k) break;
+                if (tid < 32) {  // warp 0: ballot-based compaction of the flag bits
                     int nf = 0;
-                    for (int cc = 0; cc < cx.G; ++cc)
-                        if ((s_more[cc >> 5] >> (cc & 31)) & 1u) s_flag_list[nf++] = cc;
-                    s_nflag = nf;
+                    for (int w0 = 0; w0 < (cx.G + 31) / 32; ++w0) {
+                        const int cc = w0 * 32 + tid;
+                        const bool f = cc < cx.G && ((s_more[w0] >> tid) & 1u);
+                        const uint32_t bal = __ballot_sync(0xFFFFFFFFu, f);
+                        if (f) s_flag_list[nf + __popc(bal & ((1u << tid) - 1u))] = cc;
+                        nf += __popc(bal);
+                    }
+                    if (tid == 0) s_nflag = nf;
                 }
                 CSync::sync();
             }
@@ -800,26 +808,44 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             const int span = phase == 0 ? kk : k - kk;
             const int nruns = phase == 0 ? cx.G : s_nflag;
             if (span <= 0 || nruns == 0) break;
-            const int total = nruns * span;
+            // positions q = run_slot * spanp + j with spanp = next_pow2(span): shifts, no
+            // integer division (j >= span slots are skipped)
+            const int lsp = 32 - __clz(span - 1 > 0 ? span - 1 : 0);
+            const int total = nruns << lsp;
             for (int q0 = 0; q0 < total; q0 += CI * kNC) {
                 E ents[CI];
                 uint32_t mask = 0;
+                // all loads first, unconditionally (invalid slots read entry 0 and are
+                // discarded) -- one L2 round trip instead of CI dependent ones
+                size_t at[CI];
+                bool ok[CI];
 #pragma unroll
                 for (int r = 0; r < CI; ++r) {
                     const int q = q0 + tid + r * kNC;
-                    ents[r] = E::sentinel();
-                    if (q >= total) continue;
-                    const int cc = phase == 0 ? q / span : s_flag_list[q / span];
-                    const int j = lo + q % span;
-                    if (cc == static_cast<int>(c)) continue;
-                    const E e = cand.ld(static_cast<size_t>(cc) * k + j);
-                    if (!e.is_sentinel() && !better(tb, e)) {
-                        ents[r] = e;
+                    const int qq = q < total ? q : 0;
+                    const int slot = qq >> lsp, j = qq & ((1 << lsp) - 1);
+                    const int cc = phase == 0 ? slot : s_flag_list[slot];
+                    ok[r] = q < total && j < span && cc != static_cast<int>(c);
+                    at[r] = ok[r] ? static_cast<size_t>(cc) * k + lo + j : 0;
+                }
+#pragma unroll
+                for (int r = 0; r < CI; ++r) ents[r] = cand.ld(at[r]);
+#pragma unroll
+                for (int r = 0; r < CI; ++r) {
+                    const E e = ents[r];
+                    if (ok[r] && !e.is_sentinel() && !better(tb, e)) {
                         mask |= 1u << r;
-                        if (phase == 0 && j == kk - 1 && kk < k)
+                        const int q = q0 + tid + r * kNC;
+                        const int j = lo + (q & ((1 << lsp) - 1));
+                        if (phase == 0 && j == kk - 1 && kk < k) {
+                            const int cc = q >> lsp;
                             atomicOr(&s_more[cc >> 5], 1u << (cc & 31));
+                        }
+                    } else {
+                        ents[r] = E::sentinel();
                     }
                 }
+                if (tid == 0) trace(14);
                 bool todo = true;
                 while (true) {
                     int vote = 0;
@@ -832,6 +858,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                             todo = false;
                         }
                     }
+                    if (tid == 0) trace(15);
                     if (!cbar_or(vote != 0)) break;
                     flush<Key, MIN>(buf, &st, cx, kFlushFinal);
                 }

@@ -414,7 +414,7 @@ int topk_debug_trace(int enable, uint64_t* host) {
         return -1;
     static unsigned long long zero[topk::kTraceCtas][topk::kTraceLen];
     if (cudaMemcpyToSymbol(topk::g_trace, zero, sizeof(zero)) != cudaSuccess) return -1;
-    if (cudaMemcpyToSymbol(topk::g_trace_on, &enable, sizeof(int)) != cudaSuccess) return -1;
+    if (cudaMemcpyToSymbol(topk::c_trace_on, &enable, sizeof(int)) != cudaSuccess) return -1;
     return 0;
 }
 
