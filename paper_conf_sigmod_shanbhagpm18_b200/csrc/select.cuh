@@ -31,6 +31,7 @@
 //     bounds are entries owned by some run, so a strict test against them never drops
 //     a top-k entry.
 #pragma once
+#include "cnet.cuh"
 #include "keys.cuh"
 #include "network.cuh"
 #include "ptx.cuh"
@@ -43,6 +44,9 @@ namespace topk {
 #endif
 #ifndef TOPK_STAGES
 #define TOPK_STAGES 5
+#endif
+#ifndef TOPK_LIMIT2
+#define TOPK_LIMIT2 1024  // bag limit between the boot flush and the second flush
 #endif
 #ifndef TOPK_REFRESH_AT
 #define TOPK_REFRESH_AT 12  // tile index at which warp 0 requests a rank-bound refresh
@@ -71,7 +75,8 @@ struct WsHeader {
     unsigned long long tau_g;  // max over CTAs of their k-th best
     unsigned int ticket;       // CTAs finished
     unsigned int next_tile;    // dynamic work claiming counter
-    unsigned int pad[12];
+    unsigned int npub;         // CTAs that published their boot-flush samples
+    unsigned int pad[11];
 };
 static_assert(sizeof(WsHeader) == 64, "header");
 
@@ -234,6 +239,13 @@ struct CtaState {
     unsigned long long tau_w;  // E32: the bound as one packed word
     E tau;                     // E64: the bound
     Par<E, Key> par;           // E64: fast-test parameters of tau
+    int sorted_cnt;            // cnt right after the last exact flush (bag still sorted), else -1
+    int pubd;                  // this CTA counted itself in WsHeader::npub
+    int cnt_run;               // real entries in the CTA's final run buf[0 .. K)
+    int limit;                 // bag capacity until the next flush
+    int ties;                  // a code-path stream flush could not shrink the bag
+    int wcnt[16];              // compaction: kept entries per consumer warp
+    unsigned long long own_w;  // the bag's own k-th best as a bound word (0 = none)
     unsigned long long best[kPubRows];
     uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
 };
@@ -279,7 +291,7 @@ __device__ __forceinline__ int reserve(int* cnt, int total, int limit) {
 // Returns the count before this warp's entries, or -1 if they did not fit.
 template <class E, int ITEMS>
 __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&ents)[ITEMS],
-                                      uint32_t mask, int K, int limit) {
+                                      uint32_t mask, int limit) {
     const int lane = threadIdx.x & 31;
     const int cnt = __popc(mask);
     int incl = cnt;
@@ -294,7 +306,7 @@ __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&
     if (lane == 31) old = reserve(s_cnt, total, limit);
     old = __shfl_sync(0xFFFFFFFFu, old, 31);
     if (old < 0) return -1;
-    int w = K + old + incl - cnt;
+    int w = old + incl - cnt;
 #pragma unroll
     for (int q = 0; q < ITEMS; ++q)
         if ((mask >> q) & 1u) buf.st(w++, ents[q]);
@@ -303,7 +315,7 @@ __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&
 
 // Debug counters (whole-launch totals), read with topk_debug_stats():
 // [0] flushes, [1] survivors flushed, [2] flush cycles (thread 0), [3] deferrals,
-// [4] tiles consumed, [5] refreshes.  Only rare paths touch them.
+// [4] tiles consumed, [5] refreshes, [6] exact flushes, [7] sentinel outputs (a bug).
 __device__ unsigned long long g_stats[8];
 
 // Debug timeline: per CTA up to 62 (event << 56 | globaltimer ns) stamps written by
@@ -312,6 +324,11 @@ __device__ unsigned long long g_stats[8];
 constexpr int kTraceCtas = 160, kTraceLen = 64;
 __device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
 __device__ __constant__ int c_trace_on;  // set by topk_debug_trace (constant bank: free)
+// Debug switches (topk_debug_flags): bit 0 -- no code-network path (exact flushes only);
+// bit 1 -- no boot-time wait for peers; bit 2 -- no early second flush; bit 3 -- no
+// small-buffer exact network (wnet_small); bits 4-5 -- rank-bound rows (0 = 3);
+// bits 6-7 -- second-flush limit 512 * (1 + v) (0 = TOPK_LIMIT2).
+__device__ __constant__ int c_dbg;
 __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
     unsigned long long t;
@@ -332,6 +349,8 @@ struct Ctx {
     int k, K;
     int G, gmax, J;
     int j_lo, nrows;  // rank-bound rows used: j_lo .. j_lo + nrows - 1 (t <= G)
+    int Lp;           // code network size log2 K' (K' = max(K, 16)); -1: not used (K > 512)
+    void* codes;      // shared: code-network scratch (8 x K' codes)
     bool filter;
 };
 
@@ -352,10 +371,15 @@ __device__ void rank_rows(CtaState<E, Key>* st, const Ctx& cx) {
         const unsigned long long v = cx.scratch[q];
         if (v == 0ull) continue;
         const unsigned long long* row = cx.scratch + r * cx.G;
-        int rank = 0;
+        int gt = 0, ge = 0;
 #pragma unroll 4
-        for (int c2 = 0; c2 < cx.G; ++c2) rank += row[c2] > v ? 1 : 0;
-        if (rank == t - 1) st->best[ji] = v;  // unique: samples are distinct entries
+        for (int c2 = 0; c2 < cx.G; ++c2) {
+            gt += row[c2] > v ? 1 : 0;
+            ge += row[c2] >= v ? 1 : 0;
+        }
+        // v is the t-th largest (code-only samples of different CTAs may be equal words:
+        // every thread holding that value writes the same word)
+        if (gt <= t - 1 && t - 1 < ge) st->best[ji] = v;
     }
     CSync::sync();
 }
@@ -390,53 +414,201 @@ __device__ __forceinline__ void fold_bounds(CtaState<typename KeyTraits<Key>::E,
 
 enum FlushMode { kFlushStream = 0, kFlushFinal = 1 };
 
-// Collective flush (consumers): bitonic top-K of [run | survivors | padding].
-//   stream mode: publish the run's samples and k-th best, and -- except for the very
-//   first flush, when no other CTA has published yet -- raise the bound with the rank
-//   bound over all CTAs' samples;  final mode: the network only.
+// A code as a bound word (the weakest entry with that code: index "infinity"), i.e. a
+// NON-strict bound on the code -- valid whenever >= r entries have code >= c.
+template <class E>
+__device__ __forceinline__ unsigned long long code_word(typename CodeOf<E>::C c);
+template <>
+__device__ __forceinline__ unsigned long long code_word<E32>(uint32_t c) {
+    return static_cast<unsigned long long>(c) << 32;
+}
+template <>
+__device__ __forceinline__ unsigned long long code_word<E64>(uint64_t c) {
+    return c;
+}
+
+__device__ __forceinline__ unsigned long long global_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+constexpr unsigned long long kBootWaitNs = 20000;  // cap of the boot-time wait for peers
+
+// Bound round (collective; entry after the caller's samples were stored, exit after a
+// barrier):  stream mode -- publish the bag's k-th best (tau_g), at the first flush wait
+// (bounded) until every CTA published its samples, then the rank bound over all CTAs'
+// samples;  every mode -- thread 0 folds own / tau_g / rank rows into the CTA bound.
+template <class Key, bool MIN>
+__device__ void take_bounds(CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx& cx,
+                            typename KeyTraits<Key>::E own, bool publish) {
+    if (publish) {
+        if (threadIdx.x == 0 && !own.is_sentinel()) tau_publish(cx.hdr, own);
+        if (!st->pubd && cx.G > 1 && !(c_dbg & 2)) {
+            // boot: every CTA flushes its first buffer at about the same time; wait for
+            // their samples so the very first bound is the cross-CTA rank bound (a stale
+            // or missing sample only weakens the bound -- the wait is a performance
+            // matter, never a correctness one)
+            CSync::sync();
+            if (threadIdx.x == 0) {
+                atomicAdd(&cx.hdr->npub, 1u);
+                st->pubd = 1;
+                const unsigned long long t0 = global_ns();
+                while (ld_relaxed_u32(&cx.hdr->npub) < static_cast<uint32_t>(cx.G) &&
+                       global_ns() - t0 < kBootWaitNs)
+                    __nanosleep(64);
+                __threadfence();
+            }
+            CSync::sync();
+        }
+        load_pub(cx);
+        CSync::sync();
+        rank_rows(st, cx);
+    }
+    if (threadIdx.x == 0) {
+        if (!publish)
+            for (int ji = 0; ji < kPubRows; ++ji) st->best[ji] = 0ull;
+        if (cx.filter) fold_bounds<Key, MIN>(st, cx, own);
+    }
+    CSync::sync();
+}
+
+// Keep only the bag entries not worse than tau (collective).  Every entry is read into
+// registers before a barrier, then written compacted to the front (order is
+// irrelevant: the bag is unordered).  Returns the new count (in every thread).
+template <class E>
+__device__ int compact_bag(const SBuf<E>& buf, int cnt, E tau, int* s_w) {
+    constexpr int RC = (kCap + kNC - 1) / kNC;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    E ents[RC];
+    uint32_t keep = 0;
+#pragma unroll
+    for (int q = 0; q < RC; ++q) {
+        const int e = tid + q * kNC;
+        ents[q] = e < cnt ? buf.ld(e) : E::sentinel();
+        // keep e >= tau: tau may be an entry of this very bag (its own k-th best, or
+        // its own published sample coming back through tau_g / the rank rows), and
+        // that entry can be the global k-th best
+        if (e < cnt && !better(tau, ents[q])) keep |= 1u << q;
+    }
+    const int c = __popc(keep);
+    int incl = c;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) s_w[w] = incl;
+    CSync::sync();
+    int off = 0, all = 0;
+#pragma unroll
+    for (int v = 0; v < kNC / 32; ++v) {
+        const int x = s_w[v];
+        off += v < w ? x : 0;
+        all += x;
+    }
+    int pos = off + incl - c;
+#pragma unroll
+    for (int q = 0; q < RC; ++q)
+        if ((keep >> q) & 1u) buf.st(pos++, ents[q]);
+    CSync::sync();
+    return all;
+}
+
+// Bag capacity after `nflush` flushes: right after the boot flush a small one, so that a
+// cheap second flush soon publishes samples of many more keys (the boot samples cover
+// one buffer per CTA only) and the rank bound tightens early.  A stream flush always
+// leaves at most half of the next limit (progress: a warp appends <= 512 at a time).
+__device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
+    (void)ties;
+    const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3)) : TOPK_LIMIT2;
+    return (nflush == 1 && Lp >= 0 && !(c_dbg & 4)) ? max(l2, 2 * K) : kCap;
+}
+
+// Collective flush (consumers) of the candidate bag buf[0 .. cnt):
+//   code path (filter mode, K <= 512; every stream flush, and a final flush of a large
+//     bag): the code-only network (cnet.cuh) gives the bag's k-th best code and its
+//     2^j-th best codes -> publish, bound round, drop every entry worse than the new
+//     bound.  A stream flush ends here unless ties kept the bag over half full.
+//   exact path: bitonic top-K of [bag | sentinel padding] (wnet.cuh: local sort, merge,
+//     rebuild on (code, index) entries) -> buf[0 .. K) best first; in stream mode its
+//     exact samples / k-th best are published as well.
 // Entry: barrier-consistent; exit: same.
 template <class Key, bool MIN>
 __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
                       CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx& cx,
                       FlushMode mode) {
     using E = typename KeyTraits<Key>::E;
+    using C = typename CodeOf<E>::C;
     const int k = cx.k, K = cx.K;
-    const int cnt = st->cnt;
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int c = static_cast<int>(blockIdx.x);
+    int cnt = st->cnt;
+    const int cnt0 = cnt;
     if (threadIdx.x == 0) trace(2);
     const long long t0 = clock64();
-    int P = next_pow2_i(K + cnt);
-    if (P < 2 * K) P = 2 * K;
-    for (int i = K + cnt + threadIdx.x; i < P; i += kNC) buf.st(i, E::sentinel());
-    CSync::sync();
-    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    wnet_topk<E, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
-    const E kth = buf.ld(k - 1);
     const bool publish = mode == kFlushStream && cx.filter;
-    const bool ranks = publish && st->nflush > 0;
-    if (publish) {
-        const int c = static_cast<int>(blockIdx.x);
-        if (threadIdx.x < cx.J) {
-            const E e = buf.ld((1 << threadIdx.x) - 1);
-            if (!e.is_sentinel())
-                st_relaxed_u64(cx.pub + static_cast<size_t>(threadIdx.x) * cx.gmax + c,
-                               bound_word(e));
+    bool done = false;
+    // (tie-heavy input -- a code bound cannot separate equal codes -- makes the code
+    // path useless: after it failed once, stream flushes go straight to the exact path)
+    const bool try_code = !st->ties && (publish || cnt > 2 * K);
+    bool tried = false;
+    if (cx.filter && cx.Lp >= 0 && !(c_dbg & 1) && try_code) {
+        tried = true;
+        C* S = static_cast<C*>(cx.codes);
+        cnet_topk_codes<E, kNC / 32, CSync>(buf, cnt, cx.Lp, S, w, lane);
+        if (publish && threadIdx.x < cx.J && cnt >= (1 << threadIdx.x)) {
+            st_relaxed_u64(cx.pub + static_cast<size_t>(threadIdx.x) * cx.gmax + c,
+                           code_word<E>(S[(1 << threadIdx.x) - 1]));
+            __threadfence();
         }
-        if (threadIdx.x == 0 && !kth.is_sentinel()) tau_publish(cx.hdr, kth);
-        if (ranks) {
-            load_pub(cx);
-            CSync::sync();
-            rank_rows(st, cx);
+        const E own = cnt >= k ? from_bound_word<E>(code_word<E>(S[k - 1])) : E::sentinel();
+        // half of the top K' codes equal: heavy ties (few distinct keys), which a code
+        // bound cannot separate -- finish exactly (strict (code, index) bound) at once
+        const int Kp = 1 << cx.Lp;
+        const bool heavy = cnt >= Kp && S[Kp - 1] == S[Kp / 2 - 1];
+        take_bounds<Key, MIN>(st, cx, own, publish);
+        if (!heavy) cnt = compact_bag<E>(buf, cnt, bound_get(*st), st->wcnt);
+        // a code bound that dropped less than half of a large bag is defeated by ties
+        // (equal codes): finish exactly, and skip the code path from now on
+        const bool weak = heavy || (cnt > 2 * K && 2 * cnt > cnt0);
+        done = mode == kFlushStream && !weak &&
+               cnt <= next_limit(st->nflush + 1, K, cx.Lp, 0) / 2;
+    }
+    if (!done) {
+        int P = next_pow2_i(cnt);
+        if (P < 2 * K) P = 2 * K;
+        if (P < 64) P = 64;
+        for (int i = cnt + threadIdx.x; i < P; i += kNC) buf.st(i, E::sentinel());
+        CSync::sync();
+        if (P <= 512 && !(c_dbg & 8))
+            wnet_small<E, 2, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
+        else if (P <= 1024 && !(c_dbg & 8))
+            wnet_small<E, 4, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
+        else
+            wnet_topk<E, kNC / 32, CSync>(buf, P, __ffs(K) - 1, w, lane);
+        const E kth = buf.ld(k - 1);
+        if (publish) {
+            if (threadIdx.x < cx.J) {
+                const E e = buf.ld((1 << threadIdx.x) - 1);
+                if (!e.is_sentinel())
+                    st_relaxed_u64(cx.pub + static_cast<size_t>(threadIdx.x) * cx.gmax + c,
+                                   bound_word(e));
+                __threadfence();
+            }
         }
+        take_bounds<Key, MIN>(st, cx, kth, publish);
+        if (cnt > K) cnt = K;
     }
     if (threadIdx.x == 0) {
         atomicAdd(&g_stats[0], 1ull);
-        atomicAdd(&g_stats[1], static_cast<unsigned long long>(cnt));
+        atomicAdd(&g_stats[1], static_cast<unsigned long long>(cnt0));
         atomicAdd(&g_stats[2], static_cast<unsigned long long>(clock64() - t0));
-        st->cnt = 0;
+        if (!done) atomicAdd(&g_stats[6], 1ull);
+        if (tried && !done && publish) st->ties = 1;
+        st->cnt = cnt;
+        st->sorted_cnt = done ? -1 : cnt;
         st->nflush += 1;
-        if (!ranks)
-            for (int ji = 0; ji < kPubRows; ++ji) st->best[ji] = 0ull;
-        if (cx.filter) fold_bounds<Key, MIN>(st, cx, kth);
+        st->limit = next_limit(st->nflush, K, cx.Lp, st->ties);
         st->req = 0;
         trace(3);
     }
@@ -470,7 +642,7 @@ __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
                                             const Par<typename KeyTraits<Key>::E, Key>& pr,
                                             uint32_t tlen, uint32_t lbase,
                                             const SBuf<typename KeyTraits<Key>::E>& buf,
-                                            int* s_cnt, int K, int limit) {
+                                            int* s_cnt, int limit) {
     using KT = KeyTraits<Key>;
     using E = typename KT::E;
     using Vec = typename KT::Vec;
@@ -553,7 +725,7 @@ __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
     if (lane == 31) old = reserve(s_cnt, total, limit);
     old = __shfl_sync(0xFFFFFFFFu, old, 31);
     if (old < 0) return -1;
-    int w = K + old + incl - cnt;
+    int w = old + incl - cnt;
     for (uint32_t m = keep; m; m &= m - 1u) {
         const int q = __ffs(m) - 1;
         const uint32_t pos = pos_of(q);
@@ -586,13 +758,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     const uint32_t c = blockIdx.x;
     const int K = static_cast<int>(p.K);
     const int k = static_cast<int>(p.k);
-    // Until a bound exists, keep the buffer small so the first flush is cheap.
-#ifndef TOPK_BOOT_BIG_K
-#define TOPK_BOOT_BIG_K 32
-#endif
-    // (K >= TOPK_BOOT_BIG_K: fill the whole buffer -- one larger boot flush whose run,
-    // after the rank refresh, bounds tightly enough that no second flush is needed)
-    const int boot_limit = !FILTER ? kCap - K : (K >= TOPK_BOOT_BIG_K ? kCap - K : 1024);
+    // Before the first flush every key is kept: the whole buffer is the boot sample
+    // (st.limit = kCap); after it, next_limit().
     const Key* keys = static_cast<const Key*>(p.keys);
     WsHeader* hdr = reinterpret_cast<WsHeader*>(p.ws);
     Ctx cx;
@@ -606,10 +773,14 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     cx.J = static_cast<int>(p.J);
     cx.j_lo = 0;
     while (cx.j_lo < cx.J && ((k + (1 << cx.j_lo) - 1) >> cx.j_lo) > cx.G) ++cx.j_lo;
-    cx.nrows = cx.J - cx.j_lo < 3 ? cx.J - cx.j_lo : 3;
+    {
+        const int maxrows = (c_dbg >> 4) & 3 ? (c_dbg >> 4) & 3 : 3;
+        cx.nrows = cx.J - cx.j_lo < maxrows ? cx.J - cx.j_lo : maxrows;
+    }
     cx.filter = FILTER;
+    cx.Lp = (FILTER && K <= 512) ? (K < 16 ? 4 : __ffs(K) - 1) : -1;
+    cx.codes = scratch + kScratch;
 
-    for (int i = tid; i < K; i += kNT) buf.st(i, E::sentinel());
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) {
             mbar_init(&full[s], 1);
@@ -619,6 +790,10 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         st.cnt = 0;
         st.req = 0;
         st.nflush = 0;
+        st.sorted_cnt = -1;
+        st.pubd = 0;
+        st.limit = kCap;
+        st.ties = 0;
         st.tau_w = 0ull;
         st.tau = E::sentinel();
         st.par = make_par<Key, MIN>(E::sentinel());
@@ -630,7 +805,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (tid < nextra) {
             const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
                                                                  : tail0 + (tid - p.head);
-            buf.st(K + tid, E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row)));
+            buf.st(tid, E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row)));
         }
         if (tid == 0) st.cnt = nextra;
     }
@@ -717,8 +892,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         const uint32_t lbase = static_cast<uint32_t>(p.head + tlo);
         const unsigned char* data = ring + static_cast<size_t>(slot) * kTileBytes;
         Par<E, Key> pr = load_par<Key, MIN>(st);
-        int r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, K,
-                                               pr.active ? kCap - K : boot_limit);
+        int r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, st.limit);
         while (r < 0) {  // did not fit: flush, then redo with the new bound
             if (lane == 0) {
                 atomicAdd(&g_stats[3], 1ull);
@@ -728,8 +902,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             cbar_or(true);
             collective();
             pr = load_par<Key, MIN>(st);
-            r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, K,
-                                               pr.active ? kCap - K : boot_limit);
+            r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, st.limit);
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[slot]);
@@ -739,12 +912,22 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     // Drain: serve requests of warps still streaming, until all are done.
     while (cbar_or(pending_req())) collective();
     if (tid == 0) trace(4);
-    if (tid == 0) atomicAdd(&g_stats[4], static_cast<unsigned long long>(ntiles_done));
-    if (st.cnt > 0) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
+    if (tid == 0) {
+        atomicAdd(&g_stats[4], static_cast<unsigned long long>(ntiles_done));
+        if (!st.pubd) atomicAdd(&hdr->npub, 1u);  // peers waiting at boot need not wait for us
+    }
+    // The CTA's run: the exact top-K of its bag, best first (skipped if already sorted).
+    if (st.cnt == 0) {
+        for (int j = tid; j < K; j += kNC) buf.st(j, E::sentinel());
+        CSync::sync();
+    } else if (st.cnt != st.sorted_cnt) {
+        flush<Key, MIN>(buf, &st, cx, kFlushFinal);
+    }
 
     // ---- hand the CTA's top-k to the reduction (last CTA to arrive) ----
     GBuf<E> cand;
     cand.init(p.ws + ws_cand_offset(p.gmax), static_cast<size_t>(G) * k);
+    if (tid == 0) st.cnt_run = st.cnt;
     if (G > 1) {
         for (int j = tid; j < k; j += kNC) cand.st(static_cast<size_t>(c) * k + j, buf.ld(j));
         __threadfence();
@@ -776,6 +959,15 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         }
         CSync::sync();
         const E tb = st.tau;
+        {   // own run: keep its qualifying prefix (sorted best first)
+            const int own = st.cnt_run < k ? st.cnt_run : k;
+            int q = 0;
+            for (int j = tid; j < own; j += kNC) q += better(tb, buf.ld(j)) ? 0 : 1;
+            if (q) atomicAdd(&st.cnt, q);
+            CSync::sync();
+            if (tid == 0) st.sorted_cnt = st.cnt;
+            CSync::sync();
+        }
         if (tid == 0) trace(11);
         // (2) Every run is sorted best first, so only a prefix can be >= tb: append the
         // qualifying entries of the first min(k, 32) of every other run (one parallel
@@ -851,7 +1043,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                     int vote = 0;
                     if (todo) {
                         if (__any_sync(0xFFFFFFFFu, mask != 0u)) {
-                            const int old = append<E, CI>(buf, &st.cnt, ents, mask, K, kCap - K);
+                            const int old = append<E, CI>(buf, &st.cnt, ents, mask, kCap);
                             todo = old < 0;
                             vote = todo ? 1 : 0;
                         } else {
@@ -866,11 +1058,16 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             CSync::sync();
         }
         if (tid == 0) trace(10);
-        if (st.cnt > 0) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
+        if (st.cnt != st.sorted_cnt) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
     }
     // ---- finalize: best first, original key bits, global index, payload ----
     for (int j = tid; j < k; j += kNC) {
         const E e = buf.ld(j);
+        if (e.is_sentinel()) {  // cannot happen (k <= n); never read out of bounds
+            atomicAdd(&g_stats[7], 1ull);
+            if (p.out_idx) p.out_idx[j] = -1;
+            continue;
+        }
         const uint32_t row = e.lidx();
         if (p.out_idx) p.out_idx[j] = static_cast<int64_t>(p.base + row);
         if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = keys[row];
@@ -883,6 +1080,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     if (tid == 0) {
         hdr->tau_g = 0ull;
         hdr->ticket = 0u;
+        hdr->npub = 0u;
         hdr->next_tile = 0u;
     }
 }
@@ -891,7 +1089,9 @@ template <class Key>
 constexpr size_t select_smem_bytes() {
     return static_cast<size_t>(Cfg<Key>::kStages) * kTileBytes +
            static_cast<size_t>(kCap) * SBuf<typename KeyTraits<Key>::E>::kBytes +
-           static_cast<size_t>(2 * Cfg<Key>::kStages) * 8 + static_cast<size_t>(kScratch) * 8;
+           static_cast<size_t>(2 * Cfg<Key>::kStages) * 8 + static_cast<size_t>(kScratch) * 8 +
+           static_cast<size_t>(kCap / 512) * 512 *
+               sizeof(typename CodeOf<typename KeyTraits<Key>::E>::C);  // code network
 }
 
 }  // namespace topk

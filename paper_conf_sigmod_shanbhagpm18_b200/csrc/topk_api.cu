@@ -391,8 +391,8 @@ topk_status_t topk_probe_read(const void* data, size_t bytes, int method, int gr
  * of 15 warps.  e64 selects 12-byte entries; smem_net the shared-memory network. */
 int topk_debug_netbench(int P, int L, int e64, int smem_net, int iters, uint64_t* host2) {
     unsigned long long* d = nullptr;
-    if (cudaMalloc(&d, 16) != cudaSuccess) return -1;
-    const size_t smem = 4096 * 12;
+    if (cudaMalloc(&d, 24) != cudaSuccess) return -1;
+    const size_t smem = 4096 * 12 + 4096 * 8;
     if (e64) {
         cudaFuncSetAttribute(topk::netbench_kernel<topk::E64, 15>,
                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -405,6 +405,31 @@ int topk_debug_netbench(int P, int L, int e64, int smem_net, int iters, uint64_t
     cudaError_t e = cudaMemcpy(host2, d, 16, cudaMemcpyDeviceToHost);
     cudaFree(d);
     return e == cudaSuccess ? 0 : -1;
+}
+
+/* Debug: the code-only network (cnet.cuh) on n <= 4096 device codes (u32, or u64 if
+ * e64), 4 <= Lp <= 9; d_out receives the top-2^Lp codes best first. */
+int topk_debug_cnet(int e64, const void* d_codes, int n, int Lp, void* d_out) {
+    if (n < 1 || n > 4096 || Lp < 4 || Lp > 9) return -1;
+    const size_t smem = 4096 * 12 + 4096 * 8;
+    if (e64) {
+        cudaFuncSetAttribute(topk::cnet_debug_kernel<topk::E64, 15>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        topk::cnet_debug_kernel<topk::E64, 15><<<1, 480, smem>>>(
+            static_cast<const uint64_t*>(d_codes), n, Lp, static_cast<uint64_t*>(d_out));
+    } else {
+        cudaFuncSetAttribute(topk::cnet_debug_kernel<topk::E32, 15>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        topk::cnet_debug_kernel<topk::E32, 15><<<1, 480, smem>>>(
+            static_cast<const uint32_t*>(d_codes), n, Lp, static_cast<uint32_t*>(d_out));
+    }
+    g_launches.fetch_add(1, std::memory_order_relaxed);
+    return cudaDeviceSynchronize() == cudaSuccess ? 0 : -1;
+}
+
+/* Debug switches of the select kernel (select.cuh c_dbg). */
+int topk_debug_flags(int flags) {
+    return cudaMemcpyToSymbol(topk::c_dbg, &flags, sizeof(int)) == cudaSuccess ? 0 : -1;
 }
 
 /* Debug timeline (see select.cuh g_trace): enable=1 clears and enables, 0 disables;

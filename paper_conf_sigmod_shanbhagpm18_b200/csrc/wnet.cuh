@@ -297,3 +297,110 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
 }
 
 }  // namespace topk
+
+namespace topk {
+
+// Exact bitonic top-K (K = 2^L) of a SMALL buffer b[0..P), 64 <= P <= 1024, P >= 2K --
+// the latency form used for the final flushes (a few hundred entries after the
+// code-network compaction).  All W = P / (32 R) warps keep R entries per lane for the
+// whole network; the paper's rounds of merge + rebuild (Alg. 4) do not compact
+// the survivors into fewer warps (that would serialise the rounds on one warp), the
+// discarded half just keeps computing.  Element e = w * 32R + lane * R + r: steps on
+// bits < log2 R are register compare-exchanges, the next 5 bits warp shuffles, the rest
+// exchanges through shared memory -- b[P .. 2P) and b[0 .. P) alternate, so one barrier
+// per cross-warp step suffices.  Same step semantics as wstep (Alg. 4 generalised).
+template <class E, int R, int B>
+__device__ __forceinline__ void wsmall_reg(E (&x)[R], uint32_t e0, int d) {
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+        if ((r >> B) & 1) continue;
+        constexpr int m = 1 << B;
+        const bool bf = (((e0 + r) >> d) & 1u) == 0u;
+        const E a = x[r], c = x[r | m];
+        const bool sw = bf == better(c, a);
+        x[r] = esel(sw, c, a);
+        x[r | m] = esel(sw, a, c);
+    }
+}
+
+// One step of wnet_small on element bit bb, blocks best-first iff bit d of e is 0.
+template <class E, int R, class Sync>
+__device__ __forceinline__ void wsmall_step(E (&x)[R], const SBuf<E>& b, int P, uint32_t e0,
+                                            int lane, bool act, int bb, int d, int& region) {
+    constexpr int LR = Log2<R>::v;
+    if (bb < LR) {
+        if (!act) return;
+        // compile-time register pairs (a runtime index would put x in local memory)
+        if (bb == 0) wsmall_reg<E, R, 0>(x, e0, d);
+        else if constexpr (LR > 1) wsmall_reg<E, R, 1>(x, e0, d);
+    } else if (bb < LR + 5) {
+        if (!act) return;
+        const int m = 1 << (bb - LR);
+        const bool lower = (lane & m) == 0;
+        const bool bf = ((e0 >> d) & 1u) == 0u;  // d > bb >= LR: same for every r
+        const bool keep_better = lower == bf;
+#pragma unroll
+        for (int r = 0; r < R; ++r) {
+            const E y = shfl_xor_e(x[r], m);
+            x[r] = esel(keep_better == better(y, x[r]), y, x[r]);
+        }
+    } else {
+        const int base = region * P;
+        region ^= 1;
+        if (act) {
+#pragma unroll
+            for (int r = 0; r < R; r += 2) b.st2(base + static_cast<int>(e0) + r, x[r], x[r + 1]);
+        }
+        Sync::sync();
+        if (act) {
+            const bool lower = ((e0 >> bb) & 1u) == 0u;
+            const bool bf = ((e0 >> d) & 1u) == 0u;
+            const bool keep_better = lower == bf;
+            const int pe = static_cast<int>(e0 ^ (1u << bb));
+#pragma unroll
+            for (int r = 0; r < R; r += 2) {
+                E y0, y1;
+                b.ld2(base + pe + r, y0, y1);
+                x[r] = esel(keep_better == better(y0, x[r]), y0, x[r]);
+                x[r + 1] = esel(keep_better == better(y1, x[r + 1]), y1, x[r + 1]);
+            }
+        }
+    }
+}
+
+template <class E, int R, int NW, class Sync>
+__device__ void wnet_small(const SBuf<E>& b, int P, int L, int w, int lane) {
+    const int W = P / (32 * R);
+    const bool act = w < W;
+    const uint32_t e0 = static_cast<uint32_t>(w * 32 * R + lane * R);
+    int LP = 0;
+    while ((1 << LP) < P) ++LP;
+    E x[R];
+    if (act) {
+#pragma unroll
+        for (int r = 0; r < R; r += 2) b.ld2(static_cast<int>(e0) + r, x[r], x[r + 1]);
+    }
+    int region = 1;
+#pragma unroll 1
+    for (int s = 0; s < L; ++s)
+#pragma unroll 1
+        for (int bb = s; bb >= 0; --bb)
+            wsmall_step<E, R, Sync>(x, b, P, e0, lane, act, bb, s + 1, region);
+#pragma unroll 1
+    for (int s = L; s < LP; ++s) {
+        // merge: the lower element keeps the better (bit LP of e is 0 everywhere)
+        wsmall_step<E, R, Sync>(x, b, P, e0, lane, act, s, LP, region);
+#pragma unroll 1
+        for (int bb = L - 1; bb >= 0; --bb)
+            wsmall_step<E, R, Sync>(x, b, P, e0, lane, act, bb, s + 1, region);
+    }
+    Sync::sync();  // the last exchange may still be read
+    const int K = 1 << L;
+    if (act && static_cast<int>(e0) < K) {
+#pragma unroll
+        for (int r = 0; r < R; r += 2) b.st2(static_cast<int>(e0) + r, x[r], x[r + 1]);
+    }
+    Sync::sync();
+}
+
+}  // namespace topk

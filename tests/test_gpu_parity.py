@@ -224,3 +224,34 @@ def test_chunked_device_path(cuda_device):
     r = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True,
                        text=True, timeout=600)
     assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
+
+
+@pytest.mark.parametrize("e64", [0, 1])
+@pytest.mark.parametrize("Lp", [4, 5, 6, 7, 8, 9])
+def test_code_network_order_statistics(cuda_device, e64, Lp):
+    """cnet.cuh (the code-only local sort / merge / rebuild that yields the flush bounds)
+    returns exactly the 2^Lp largest codes, best first (positions past n count as 0):
+    the definition is a descending sort of the codes."""
+    import ctypes
+    from paper_conf_sigmod_shanbhagpm18_b200 import _lib
+    lib = _lib.load()
+    lib.topk_debug_cnet.argtypes = [ctypes.c_int, ctypes.c_void_p, ctypes.c_int, ctypes.c_int,
+                                    ctypes.c_void_p]
+    rng = np.random.default_rng(1000 + 10 * Lp + e64)
+    dt = np.uint64 if e64 else np.uint32
+    hi = np.iinfo(dt).max
+    Kp = 1 << Lp
+    for n in (1, 17, 100, 511, 512, 513, 1000, 2048, 3840, 4096):
+        cases = [rng.integers(0, hi, n, dtype=dt, endpoint=True),
+                 (rng.integers(0, 7, n) * (hi // 7)).astype(dt),          # heavy ties
+                 np.arange(n, dtype=dt), np.arange(n, dtype=dt)[::-1].copy(),
+                 rng.integers(0, 2, n).astype(dt)]                         # 0/1 principle
+        for codes in cases:
+            d = torch.from_numpy(codes.view(np.int64 if e64 else np.int32)).to(cuda_device)
+            out = torch.empty(Kp, dtype=torch.int64 if e64 else torch.int32, device=cuda_device)
+            assert lib.topk_debug_cnet(e64, d.data_ptr(), n, Lp, out.data_ptr()) == 0
+            got = out.cpu().numpy().view(dt)
+            want = np.zeros(Kp, dtype=dt)
+            srt = np.sort(codes)[::-1][:Kp]
+            want[:len(srt)] = srt
+            assert np.array_equal(got, want), (n, Lp, e64, got[:8], want[:8])
