@@ -179,11 +179,15 @@ def run_ours(args):
     out_v = torch.empty(k, dtype=torch.float32, device=dev)
     out_i = torch.empty(k, dtype=torch.int64, device=dev)
 
-    from paper_conf_sigmod_shanbhagpm18_b200.dist import sharded_topk
+    from paper_conf_sigmod_shanbhagpm18_b200.dist import NcclComm, sharded_topk_native
+
+    comm = NcclComm(device=dev) if world > 1 else None
 
     def step():
-        if world > 1:  # local top-k (base = shard offset) + NCCL all-gather + merge kernel
-            return sharded_topk(x, k, True, base=rank * n)
+        if world > 1:  # C ABI topk_select_sharded: local top-k (base = shard offset) ->
+            # ncclAllGather of the k candidates -> merge kernel, one stream, no host sync
+            return sharded_topk_native(x, k, comm, True, base=rank * n,
+                                       out=(out_v, out_i, None))
         return tk.topk(x, k, True, base=rank * n, out=(out_v, out_i, None))
 
     for _ in range(max(3, args.warmup)):
@@ -219,7 +223,7 @@ def run_ours(args):
 
     def e2e_step_sharded():
         xd.copy_(hx, non_blocking=True)
-        v, i = sharded_topk(xd, k, True, base=rank * n)
+        v, i = sharded_topk_native(xd, k, comm, True, base=rank * n, out=(out_v, out_i, None))
         hv.copy_(v, non_blocking=True)
         hi.copy_(i, non_blocking=True)
 
@@ -340,6 +344,7 @@ def run_ours(args):
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier()
+        comm.close()
         dist.destroy_process_group()
 
 

@@ -55,7 +55,8 @@ typedef enum {
     TOPK_ERR_INVALID_ARG = 1, /* NULL input, k == 0, k > n, k > 1024, bad enum, alias  */
     TOPK_ERR_UNSUPPORTED = 2, /* device is not sm_100 (B200)                          */
     TOPK_ERR_WORKSPACE = 3,   /* ws NULL, too small or misaligned                      */
-    TOPK_ERR_CUDA = 4         /* a CUDA runtime call or kernel launch failed           */
+    TOPK_ERR_CUDA = 4,        /* a CUDA runtime call or kernel launch failed           */
+    TOPK_ERR_NCCL = 5         /* an NCCL call failed (sharded entry points)            */
 } topk_status_t;
 
 typedef enum {
@@ -143,6 +144,42 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
                          uint32_t k, topk_order_t order, void* out_keys,
                          uint32_t* out_payload, int64_t* out_idx, void* ws,
                          size_t ws_bytes, void* stream);
+
+/* ---- Multi-GPU: the partitioned top-k (§1 "per-partition top-k ... global top-k
+ * from the m per-partition heaps"; App. C "combined in a final global step") ----
+ * One process (or thread) per GPU; rank r holds the global rows [base, base + n_local)
+ * of the input.  topk_select_sharded runs, enqueued on `stream`:
+ *   (1) the local top-k of keys[0 .. n_local) (topk_select, ids base + i),
+ *   (2) ncclAllGather of the k (key, int64 id[, uint32 payload]) candidates of every
+ *       rank over `comm` (NVLink / NVSwitch),
+ *   (3) topk_merge of the nranks * k candidates -- the exact global top-k, ties to the
+ *       lowest GLOBAL id, identical on every rank.
+ * Collective: every rank of `comm` must call it with the same k and order (and all with
+ * or all without payload).  n_local >= k on every rank; nranks * k <= 65536.
+ * comm is an ncclComm_t (as void*) -- made with topk_nccl_comm_init, or any NCCL
+ * communicator of the same NCCL library.  ws: DEVICE workspace of
+ * topk_sharded_workspace_bytes(...) bytes, 256-byte aligned, zero-filled before first
+ * use (topk_workspace_init).  Outputs are DEVICE pointers (k entries, any may be NULL).
+ * NCCL is loaded at run time (libnccl.so.2; the copy already in the process if any):
+ * TOPK_ERR_UNSUPPORTED if it cannot be found, TOPK_ERR_NCCL if a call fails. */
+#define TOPK_NCCL_UNIQUE_ID_BYTES 128
+/* ncclGetUniqueId into id[128] (host memory), to be broadcast to every rank. */
+topk_status_t topk_nccl_unique_id(void* id);
+/* ncclCommInitRank(comm, nranks, id, rank); *comm receives the ncclComm_t.  The calling
+ * thread's current CUDA device is the rank's device.  Collective over the ranks. */
+topk_status_t topk_nccl_comm_init(const void* id, int nranks, int rank, void** comm);
+topk_status_t topk_nccl_comm_destroy(void* comm);
+size_t topk_sharded_workspace_bytes(topk_dtype_t dtype, uint64_t n_local, uint32_t k,
+                                    int nranks);
+topk_status_t topk_select_sharded(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
+                                  uint64_t n_local, uint64_t base, uint32_t k,
+                                  topk_order_t order, void* out_keys, uint32_t* out_payload,
+                                  int64_t* out_idx, void* comm, void* ws, size_t ws_bytes,
+                                  void* stream);
+/* f32 convenience. */
+topk_status_t topk_f32_sharded(const float* keys, uint64_t n_local, uint64_t base, uint32_t k,
+                               topk_order_t order, float* out_keys, int64_t* out_idx, void* comm,
+                               void* ws, size_t ws_bytes, void* stream);
 
 /* Read-bandwidth probe (the paper's "Memory Bandwidth" line: the time to read
  * the data once, a lower bound for any top-k): reads `bytes` (multiple of 16, 16-byte

@@ -13,7 +13,7 @@ from . import _build
 
 TOPK_OK = 0
 STATUS = {0: "TOPK_OK", 1: "TOPK_ERR_INVALID_ARG", 2: "TOPK_ERR_UNSUPPORTED",
-          3: "TOPK_ERR_WORKSPACE", 4: "TOPK_ERR_CUDA"}
+          3: "TOPK_ERR_WORKSPACE", 4: "TOPK_ERR_CUDA", 5: "TOPK_ERR_NCCL"}
 F32, U32, F64 = 0, 1, 2
 LARGEST, SMALLEST = 0, 1
 MODE_FILTER, MODE_PURE = 0, 1
@@ -23,7 +23,9 @@ SYMBOLS = (
     "topk_workspace_bytes", "topk_workspace_init", "topk_select", "topk_f32", "topk_u32",
     "topk_f64", "topk_u32_kv", "topk_f64_kv", "topk_merge_workspace_bytes", "topk_merge",
     "topk_launch_count", "topk_status_string", "topk_abi_version", "topk_probe_read",
-    "topk_host_workspace_bytes", "topk_select_host",
+    "topk_host_workspace_bytes", "topk_select_host", "topk_nccl_unique_id", "topk_nccl_comm_init",
+    "topk_nccl_comm_destroy", "topk_sharded_workspace_bytes", "topk_select_sharded",
+    "topk_f32_sharded",
 )
 
 _lib = None
@@ -70,6 +72,19 @@ def load(build_if_missing: bool = True):
     lib.topk_host_workspace_bytes.restype = sz
     lib.topk_select_host.argtypes = [i32, vp, u64, u32, i32, vp, vp, u64, vp, sz, vp]
     lib.topk_select_host.restype = i32
+    lib.topk_nccl_unique_id.argtypes = [vp]
+    lib.topk_nccl_unique_id.restype = i32
+    lib.topk_nccl_comm_init.argtypes = [vp, i32, i32, ctypes.POINTER(ctypes.c_void_p)]
+    lib.topk_nccl_comm_init.restype = i32
+    lib.topk_nccl_comm_destroy.argtypes = [vp]
+    lib.topk_nccl_comm_destroy.restype = i32
+    lib.topk_sharded_workspace_bytes.argtypes = [i32, u64, u32, i32]
+    lib.topk_sharded_workspace_bytes.restype = sz
+    lib.topk_select_sharded.argtypes = [i32, vp, vp, u64, u64, u32, i32, vp, vp, vp, vp, vp, sz,
+                                        vp]
+    lib.topk_select_sharded.restype = i32
+    lib.topk_f32_sharded.argtypes = [vp, u64, u64, u32, i32, vp, vp, vp, vp, sz, vp]
+    lib.topk_f32_sharded.restype = i32
     lib.topk_launch_count.argtypes = []
     lib.topk_launch_count.restype = u64
     lib.topk_status_string.argtypes = [i32]

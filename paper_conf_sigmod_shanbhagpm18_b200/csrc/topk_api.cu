@@ -549,6 +549,7 @@ const char* topk_status_string(topk_status_t s) {
         case TOPK_ERR_UNSUPPORTED: return "TOPK_ERR_UNSUPPORTED: device or size not supported";
         case TOPK_ERR_WORKSPACE: return "TOPK_ERR_WORKSPACE: workspace NULL, too small or misaligned";
         case TOPK_ERR_CUDA: return "TOPK_ERR_CUDA: CUDA runtime or launch error";
+        case TOPK_ERR_NCCL: return "TOPK_ERR_NCCL: NCCL call failed";
     }
     return "unknown topk_status_t";
 }
@@ -588,3 +589,5 @@ static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
     }
     return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
 }
+
+#include "sharded.cuh"

@@ -55,3 +55,79 @@ def sharded_topk(x_local: torch.Tensor, k: int, largest: bool = True, base: int 
     dist.all_gather_into_tensor(gv, v, group=group)
     dist.all_gather_into_tensor(gi, i, group=group)
     return merge_fn(gv, gi, k, largest, world)
+
+
+class NcclComm:
+    """An NCCL communicator owned by the C ABI (topk_nccl_comm_init) for
+    topk_select_sharded.  Rank 0 makes the unique id; it reaches the other ranks through
+    ``group`` (any torch.distributed backend -- only the 128-byte id travels there)."""
+
+    def __init__(self, group=None, device=None):
+        import ctypes
+        from . import _lib
+        lib = _lib.load()
+        on = dist.is_available() and dist.is_initialized()
+        self.rank = dist.get_rank(group) if on else 0
+        self.world = dist.get_world_size(group) if on else 1
+        self.device = torch.device("cuda", torch.cuda.current_device()) if device is None \
+            else torch.device(device)
+        uid = ctypes.create_string_buffer(128)
+        if self.rank == 0:
+            _lib.check(lib.topk_nccl_unique_id(uid), "topk_nccl_unique_id")
+        obj = [bytes(uid.raw)]
+        if self.world > 1:
+            dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0)
+                                       if group is not None else 0, group=group)
+        uid = ctypes.create_string_buffer(obj[0], 128)
+        comm = ctypes.c_void_p()
+        with torch.cuda.device(self.device):
+            _lib.check(lib.topk_nccl_comm_init(uid, self.world, self.rank, ctypes.byref(comm)),
+                       "topk_nccl_comm_init")
+        self.ptr = comm
+        self._ws = None
+
+    def workspace(self, dtype_code: int, n_local: int, k: int):
+        from . import _lib
+        from . import Workspace
+        need = int(_lib.load().topk_sharded_workspace_bytes(dtype_code, n_local, k, self.world))
+        if need == 0:
+            raise _lib.TopkError(f"invalid sharded arguments (n_local={n_local}, k={k})")
+        if self._ws is None or self._ws.nbytes < need:
+            self._ws = Workspace(need, self.device)
+        return self._ws
+
+    def close(self):
+        from . import _lib
+        if self.ptr:
+            _lib.load().topk_nccl_comm_destroy(self.ptr)
+            self.ptr = None
+
+
+def sharded_topk_native(x_local: torch.Tensor, k: int, comm: NcclComm, largest: bool = True,
+                        base: int = 0, payload: torch.Tensor | None = None, out=None):
+    """Exact top-k of the union of every rank's shard through the C ABI's
+    topk_select_sharded: local select kernel -> ncclAllGather of the k candidates ->
+    merge kernel, all enqueued on the current stream (no host synchronisation).
+    Returns (values, int64 global ids[, payload]) on every rank."""
+    import ctypes
+    from . import _lib, _dtype_code, _ptr, _stream_ptr
+    if not x_local.is_cuda or x_local.dim() != 1:
+        raise ValueError("sharded_topk_native expects a 1-D CUDA tensor")
+    lib = _lib.load()
+    dt = _dtype_code(x_local)
+    n = x_local.shape[0]
+    x_local = x_local.contiguous()
+    if out is None:
+        vals = torch.empty(k, dtype=x_local.dtype, device=x_local.device)
+        idx = torch.empty(k, dtype=torch.int64, device=x_local.device)
+        pay = torch.empty(k, dtype=torch.uint32, device=x_local.device) \
+            if payload is not None else None
+    else:
+        vals, idx, pay = out
+    ws = comm.workspace(dt, n, k)
+    st = lib.topk_select_sharded(dt, _ptr(x_local), _ptr(payload), n, base, k,
+                                 _lib.LARGEST if largest else _lib.SMALLEST, _ptr(vals),
+                                 _ptr(pay), _ptr(idx), comm.ptr, ws.ptr(), ws.nbytes,
+                                 _stream_ptr(x_local.device))
+    _lib.check(st, "topk_select_sharded")
+    return (vals, idx) if payload is None else (vals, idx, pay)

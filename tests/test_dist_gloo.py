@@ -75,3 +75,61 @@ def test_sharded_topk_world2_gloo():
             vb, il = out[r][ci]
             assert il == oi.tolist(), (dname, r)
             assert vb == ov.tobytes()
+
+
+def _comm_worker(rank, world, port, q):
+    """NcclComm's host logic: rank 0's unique id reaches every rank through the torch
+    group and each rank initialises its communicator with (id, world, rank).  The two
+    C calls are replaced by recorders (no GPU / NCCL here)."""
+    import ctypes
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    from paper_conf_sigmod_shanbhagpm18_b200 import _lib, dist as tkdist
+
+    calls = []
+
+    class FakeLib:
+        def topk_nccl_unique_id(self, buf):
+            ctypes.memmove(buf, bytes(range(7, 7 + 128)), 128)
+            return 0
+
+        def topk_nccl_comm_init(self, uid, nranks, r, out):
+            calls.append((bytes(uid.raw), nranks, r))
+            return 0
+
+    _lib.load = lambda build_if_missing=True: FakeLib()
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+
+    class _Dev:  # torch.cuda.device(...) needs no GPU for this check
+        def __init__(self, *a):
+            pass
+
+        def __enter__(self):
+            return self
+
+        def __exit__(self, *a):
+            return False
+
+    torch.cuda.device = _Dev
+    tkdist.NcclComm(device="cpu")
+    q.put((rank, calls))
+    dist.destroy_process_group()
+
+
+def test_nccl_comm_id_broadcast_world2_gloo():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_comm_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=180) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    want = bytes(range(7, 7 + 128))
+    for r in range(2):
+        assert out[r] == [(want, 2, r)]

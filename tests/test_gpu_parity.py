@@ -255,3 +255,26 @@ def test_code_network_order_statistics(cuda_device, e64, Lp):
             srt = np.sort(codes)[::-1][:Kp]
             want[:len(srt)] = srt
             assert np.array_equal(got, want), (n, Lp, e64, got[:8], want[:8])
+
+
+@pytest.mark.parametrize("dt", ["f32", "u32", "f64"])
+def test_sharded_c_abi_one_rank(cuda_device, dt):
+    """topk_select_sharded (local select -> ncclAllGather -> merge kernel) over a real
+    one-rank NCCL communicator: global ids = base + i, bit-exact vs the oracle."""
+    from paper_conf_sigmod_shanbhagpm18_b200.dist import NcclComm, sharded_topk_native
+    comm = NcclComm(device=cuda_device)
+    try:
+        n, base = (1 << 20) + 7, 5 << 30
+        x = datagen.generate("uniform", n, dt, seed=606)
+        p = datagen.payload(n, seed=606)
+        keys = host(x)
+        for k, largest in ((1, True), (64, False), (1000, True)):
+            v, i, pv = sharded_topk_native(x.to(cuda_device), k, comm, largest, base=base,
+                                           payload=p.to(cuda_device))
+            torch.cuda.synchronize()
+            ov, oi = oracle.topk(keys, k, largest, base=base)
+            assert np.array_equal(i.cpu().numpy(), oi)
+            assert host(v).tobytes() == ov.tobytes()
+            assert np.array_equal(host(pv), host(p)[oi - base])
+    finally:
+        comm.close()
