@@ -316,19 +316,19 @@ __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&
 // Debug counters (whole-launch totals), read with topk_debug_stats():
 // [0] flushes, [1] survivors flushed, [2] flush cycles (thread 0), [3] deferrals,
 // [4] tiles consumed, [5] refreshes, [6] exact flushes, [7] sentinel outputs (a bug).
-__device__ unsigned long long g_stats[8];
+static __device__ unsigned long long g_stats[8];  // per translation unit (select_tu.cuh)
 
 // Debug timeline: per CTA up to 62 (event << 56 | globaltimer ns) stamps written by
 // consumer thread 0 (events: 1 start, 2 flush begin, 3 flush end, 4 stream end,
 // 5 tail begin, 6 end, 7 refresh); g_trace[c][0] = count.  Enabled by g_trace_on.
 constexpr int kTraceCtas = 160, kTraceLen = 64;
-__device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
-__device__ __constant__ int c_trace_on;  // set by topk_debug_trace (constant bank: free)
+static __device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
+static __device__ __constant__ int c_trace_on;  // set by topk_debug_trace (constant bank: free)
 // Debug switches (topk_debug_flags): bit 0 -- no code-network path (exact flushes only);
 // bit 1 -- no boot-time wait for peers; bit 2 -- no early second flush; bit 3 -- no
 // small-buffer exact network (wnet_small); bits 4-5 -- rank-bound rows (0 = 3);
 // bits 6-7 -- second-flush limit 512 * (1 + v) (0 = TOPK_LIMIT2).
-__device__ __constant__ int c_dbg;
+static __device__ __constant__ int c_dbg;
 __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
     unsigned long long t;

@@ -11,6 +11,7 @@
 #include "merge.cuh"
 #include "probe.cuh"
 #include "netbench.cuh"
+#include "dispatch.h"
 #include "select.cuh"
 #include "topk.h"
 
@@ -60,31 +61,21 @@ bool valid_order(int o) { return o == TOPK_LARGEST || o == TOPK_SMALLEST; }
 // the sentinel entry).
 constexpr uint64_t kMaxLaunchN = 0xFFFFFFFEull;
 
-template <class Key, bool MIN, bool FILTER>
-cudaError_t launch_select(const topk::SelectParams& p, int grid, cudaStream_t st) {
-    static bool attr_set = false;  // per instantiation (benign race: idempotent)
-    const size_t smem = topk::select_smem_bytes<Key>();
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(topk::select_kernel<Key, MIN, FILTER>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(smem));
-        if (e != cudaSuccess) return e;
-        attr_set = true;
+cudaError_t dispatch_select(topk_dtype_t dt, const topk::SelectParams& p, int grid,
+                            bool min_order, bool filter, cudaStream_t st) {
+    cudaError_t e;
+    switch (dt) {
+        case TOPK_F32: e = topk::launch_select_f32(p, grid, min_order, filter, st); break;
+        case TOPK_U32: e = topk::launch_select_u32(p, grid, min_order, filter, st); break;
+        default: e = topk::launch_select_f64(p, grid, min_order, filter, st); break;
     }
-    topk::select_kernel<Key, MIN, FILTER><<<grid, topk::kNT, smem, st>>>(p);
-    g_launches.fetch_add(1, std::memory_order_relaxed);
-    return cudaGetLastError();
+    if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
+    return e;
 }
 
-template <class Key>
-cudaError_t dispatch_select(const topk::SelectParams& p, int grid, bool min_order, bool filter,
-                            cudaStream_t st) {
-    if (min_order)
-        return filter ? launch_select<Key, true, true>(p, grid, st)
-                      : launch_select<Key, true, false>(p, grid, st);
-    return filter ? launch_select<Key, false, true>(p, grid, st)
-                  : launch_select<Key, false, false>(p, grid, st);
-}
+// Every select translation unit's debug accessor (each holds its own device globals).
+int (*const kSelectDebug[])(int, void*, int) = {topk::debug_select_f32, topk::debug_select_u32,
+                                                topk::debug_select_f64};
 
 template <class Key, bool MIN>
 cudaError_t launch_merge(const topk::MergeParams& p, cudaStream_t st) {
@@ -245,13 +236,7 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
-    cudaError_t e;
-    switch (dtype) {
-        case TOPK_F32: e = dispatch_select<float>(p, grid, mn, filt, st); break;
-        case TOPK_U32: e = dispatch_select<uint32_t>(p, grid, mn, filt, st); break;
-        default: e = dispatch_select<double>(p, grid, mn, filt, st); break;
-    }
-    return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+    return dispatch_select(dtype, p, grid, mn, filt, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
 }
 
 
@@ -350,11 +335,10 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
 /* Debug (not in topk.h's stable surface): read / reset the device counters of
  * select_kernel (flushes, survivors flushed, flush cycles, deferrals, tiles). */
 int topk_debug_stats(uint64_t* host8, int reset) {
-    if (cudaMemcpyFromSymbol(host8, topk::g_stats, sizeof(unsigned long long) * 8) != cudaSuccess)
-        return -1;
-    if (reset) {
-        unsigned long long z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-        if (cudaMemcpyToSymbol(topk::g_stats, z, sizeof(z)) != cudaSuccess) return -1;
+    for (int i = 0; i < 8; ++i) host8[i] = 0;
+    for (auto f : kSelectDebug) {
+        if (f(topk::kDbgStatsAdd, host8, 0) != 0) return -1;
+        if (reset && f(topk::kDbgStatsReset, nullptr, 0) != 0) return -1;
     }
     return 0;
 }
@@ -427,19 +411,30 @@ int topk_debug_cnet(int e64, const void* d_codes, int n, int Lp, void* d_out) {
     return cudaDeviceSynchronize() == cudaSuccess ? 0 : -1;
 }
 
-/* Debug switches of the select kernel (select.cuh c_dbg). */
+/* Debug switches of the select kernel (select.cuh c_dbg), set in every select TU. */
 int topk_debug_flags(int flags) {
-    return cudaMemcpyToSymbol(topk::c_dbg, &flags, sizeof(int)) == cudaSuccess ? 0 : -1;
+    for (auto f : kSelectDebug)
+        if (f(topk::kDbgFlags, nullptr, flags) != 0) return -1;
+    return 0;
 }
 
 /* Debug timeline (see select.cuh g_trace): enable=1 clears and enables, 0 disables;
- * copies kTraceCtas x kTraceLen u64 to host (may be NULL). */
+ * copies kTraceCtas x kTraceLen u64 to host (may be NULL) -- per CTA row, from the
+ * select TU that recorded events (one key type is traced at a time). */
 int topk_debug_trace(int enable, uint64_t* host) {
-    if (host && cudaMemcpyFromSymbol(host, topk::g_trace, sizeof(topk::g_trace)) != cudaSuccess)
-        return -1;
-    static unsigned long long zero[topk::kTraceCtas][topk::kTraceLen];
-    if (cudaMemcpyToSymbol(topk::g_trace, zero, sizeof(zero)) != cudaSuccess) return -1;
-    if (cudaMemcpyToSymbol(topk::c_trace_on, &enable, sizeof(int)) != cudaSuccess) return -1;
+    constexpr size_t kRows = topk::kTraceCtas, kLen = topk::kTraceLen;
+    if (host) {
+        static uint64_t tmp[kRows * kLen];
+        std::memset(host, 0, sizeof(tmp));
+        for (auto f : kSelectDebug) {
+            if (f(topk::kDbgTraceRead, tmp, 0) != 0) return -1;
+            for (size_t r = 0; r < kRows; ++r)
+                if (tmp[r * kLen] > host[r * kLen])
+                    std::memcpy(host + r * kLen, tmp + r * kLen, kLen * sizeof(uint64_t));
+        }
+    }
+    for (auto f : kSelectDebug)
+        if (f(topk::kDbgTraceSet, nullptr, enable) != 0) return -1;
     return 0;
 }
 

@@ -25,7 +25,7 @@
 namespace topk {
 
 // netbench instrumentation: clock64 at the end of phase A of the last network call
-__device__ long long g_wnet_phase_a_end;
+static __device__ long long g_wnet_phase_a_end;  // per translation unit
 
 template <class E>
 __device__ __forceinline__ E shfl_xor_e(const E& e, int m);
