@@ -33,7 +33,8 @@ _lib = None
 def build(force: bool = False) -> str:
     """Compile the oracle with g++ (no CUDA).  Building the checker is not using it."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-shared", "-fPIC", "-pthread",
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-shared",
+                               "-fPIC", "-pthread",
                                "-o", _LIB, _SRC])
     return _LIB
 
@@ -50,6 +51,9 @@ def _load():
         lib.oracle_certificate.restype = i32
         lib.oracle_codes.argtypes = [i32, vp, u64, i32, vp]
         lib.oracle_codes.restype = None
+        lib.oracle_query.argtypes = [i32, vp, vp, ctypes.c_float, i32, vp, u32, u32, u64, u64,
+                                     u32, i32, vp, vp, i32]
+        lib.oracle_query.restype = i32
         lib.oracle_threads.argtypes = []
         lib.oracle_threads.restype = i32
         _lib = lib
@@ -80,6 +84,45 @@ def topk(keys: np.ndarray, k: int, largest: bool = True, base: int = 0,
     if r < 0:
         raise ValueError(f"oracle_topk: invalid arguments (n={n}, k={k})")
     return out_k, out_i
+
+
+PRED_NONE, PRED_RANGE, PRED_IN = 0, 1, 2
+
+
+def query(keys: np.ndarray, k: int, largest: bool = True, rank_b: np.ndarray | None = None,
+          rank_w: float = 0.0, pred: tuple | None = None, threads: int = 0):
+    """``SELECT WHERE pred ORDER BY f LIMIT k`` (R17/R18).
+
+    ``pred``: None, ``("range", col_u32, lo, hi)`` (lo <= col < hi) or
+    ``("in", col_u32, mask64)`` (col < 64 and bit col of mask).  ``rank_b``: None
+    (f = keys) or a float32 column (f = keys + rank_w * rank_b, each op rounded to f32).
+    Returns ``(values, indices, m)``: m = result rows (<= k); rows j >= m have index -1
+    and zero key bits.
+    """
+    keys = np.ascontiguousarray(keys)
+    dt = _NP2DT[keys.dtype]
+    n = keys.shape[0]
+    kind, col, lo, hi, mask = PRED_NONE, None, 0, 0, 0
+    if pred is not None:
+        if pred[0] == "range":
+            kind, col, lo, hi = PRED_RANGE, pred[1], int(pred[2]), int(pred[3])
+        elif pred[0] == "in":
+            kind, col, mask = PRED_IN, pred[1], int(pred[2])
+        else:
+            raise ValueError(pred[0])
+        col = np.ascontiguousarray(col, dtype=np.uint32)
+        assert col.shape[0] == n
+    if rank_b is not None:
+        rank_b = np.ascontiguousarray(rank_b, dtype=np.float32)
+        assert rank_b.shape[0] == n
+    out_k = np.empty(k, dtype=keys.dtype)
+    out_i = np.empty(k, dtype=np.int64)
+    m = _load().oracle_query(dt, _ptr(keys), _ptr(rank_b), float(rank_w), kind, _ptr(col),
+                             lo, hi, mask, n, k, 0 if largest else 1, _ptr(out_k), _ptr(out_i),
+                             threads)
+    if m < 0:
+        raise ValueError("oracle_query: invalid arguments")
+    return out_k, out_i, m
 
 
 def certificate(keys: np.ndarray, k: int, out_keys: np.ndarray, out_idx: np.ndarray,

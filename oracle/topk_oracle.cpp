@@ -26,7 +26,12 @@
  * std::partial_sort's its chunk to its best k; one final std::partial_sort over the
  * P*k winners.  Exact because top-k decomposes under a strict total order.
  *
- * Also: oracle_certificate(), an O(n) check independent of partial_sort.
+ * Also: oracle_certificate(), an O(n) check independent of partial_sort,
+ * and oracle_query(), the database form of §5: WHERE predicate, ORDER BY a
+ * ranking function, LIMIT k -- computed the unfused way the paper starts from ("a
+ * separate kernel execute[s] the filter and ... the subsequent top-k kernel use[s] the
+ * output"; "a separate projection step which outputs the value of the
+ * function"): filter rows, project f, then the top-k above.
  */
 #include <algorithm>
 #include <cmath>
@@ -199,6 +204,56 @@ int oracle_certificate(int dtype, const void* keys, uint64_t n, uint64_t base, u
         if (better(p, last)) ++cnt;
     }
     return cnt == (uint64_t)(k - 1) ? 0 : 3;
+}
+
+/* Query form (queries 1-3 of §6.8):
+ *   SELECT row, f(row) WHERE pred(row) ORDER BY f DESC|ASC LIMIT k
+ * pred (reading R17): kind 0 none; 1 range lo <= pcol[i] < hi; 2 membership
+ *   pcol[i] < 64 and bit pcol[i] of in_mask set (an IN list over a dictionary-coded
+ *   column, e.g. "lang = 'en' OR lang = 'es'").
+ * f (reading R18): rank_b == NULL -> f = keys[i] (any dtype); else (f32 only)
+ *   f = keys[i] + w * rank_b[i], the product and the sum each rounded to float
+ *   ("retweet_count + 0.5 * likes_count"; built with -ffp-contract=off).
+ * Plain plan: (1) filter + project into a new array with the source row ids, (2)
+ * oracle_topk over it with explicit indices.  Rows beyond the number of matches get
+ * out_idx = -1 and all-zero key bits.  Returns the number of result rows (<= k), or
+ * -1 on an argument error. */
+int oracle_query(int dtype, const void* keys, const float* rank_b, float w, int pred_kind,
+                 const uint32_t* pcol, uint32_t lo, uint32_t hi, uint64_t in_mask, uint64_t n,
+                 uint32_t k, int order, void* out_keys, int64_t* out_idx, int threads) {
+    if (!keys || n == 0 || k == 0 || dtype < 0 || dtype > 2) return -1;
+    if (rank_b && dtype != DT_F32) return -1;
+    if (pred_kind < 0 || pred_kind > 2 || (pred_kind && !pcol)) return -1;
+    const size_t kb = key_bytes(dtype);
+    std::vector<unsigned char> fk;
+    std::vector<int64_t> fi;
+    fk.reserve(n * kb);
+    fi.reserve(n);
+    for (uint64_t i = 0; i < n; ++i) {
+        if (pred_kind == 1 && !(lo <= pcol[i] && pcol[i] < hi)) continue;
+        if (pred_kind == 2 && !(pcol[i] < 64 && ((in_mask >> pcol[i]) & 1ull))) continue;
+        unsigned char b[8];
+        if (rank_b) {
+            float a;
+            std::memcpy(&a, static_cast<const char*>(keys) + 4 * i, 4);
+            const float prod = w * rank_b[i];
+            const float f = a + prod;
+            std::memcpy(b, &f, 4);
+        } else {
+            std::memcpy(b, static_cast<const char*>(keys) + kb * i, kb);
+        }
+        fk.insert(fk.end(), b, b + kb);
+        fi.push_back(static_cast<int64_t>(i));
+    }
+    const uint64_t m = fi.size();
+    const uint32_t kk = m < k ? static_cast<uint32_t>(m) : k;
+    if (out_keys) std::memset(out_keys, 0, kb * k);
+    if (out_idx)
+        for (uint32_t j = 0; j < k; ++j) out_idx[j] = -1;
+    if (kk > 0 && oracle_topk(dtype, fk.data(), fi.data(), m, 0, kk, order, out_keys, out_idx,
+                              threads) < 0)
+        return -1;
+    return static_cast<int>(kk);
 }
 
 /* Order code of each key (exposed so tests can pin the code map itself against
