@@ -115,6 +115,43 @@ topk_status_t topk_f64_kv(const double* keys, const uint32_t* payload, uint64_t 
                           uint32_t* out_payload, int64_t* out_idx, void* ws,
                           size_t ws_bytes, void* stream);
 
+/* ---- Query form: the paper's §5 database integration ----
+ *   SELECT row WHERE pred(row) ORDER BY f(row) DESC|ASC LIMIT k
+ * "Fusing with filter": the predicate runs inside the streaming pass as the
+ * FusedSortReducer's buffer filler -- a row enters the shared-memory buffer only if it
+ * matches (and can still be in the top-k); nothing filtered is written to memory.
+ * "Custom ranking function": f(A1, A2) is evaluated inside the same pass
+ * instead of a separate projection.  Queries 1-3 of §6.8 have this shape.
+ *   pred   NULL (no WHERE) or a topk_pred_t:
+ *            TOPK_PRED_RANGE  lo <= col[i] < hi            ("tweet_time < X")
+ *            TOPK_PRED_IN     col[i] < 64 and bit col[i] of in_mask set -- an IN list
+ *                             over a dictionary-coded column ("lang='en' OR lang='es'",
+ *                             P:300)
+ *          col is a DEVICE uint32 column [n].
+ *   rank_b NULL: f = keys[i] (dtype F32 / U32 / F64).  Otherwise (dtype F32 only) the
+ *          ranking function f = keys[i] + rank_w * rank_b[i], the product and the sum
+ *          each rounded to nearest float ("retweet_count + 0.5 * likes_count");
+ *          rank_b is a DEVICE float column [n].
+ *   Result: out_keys[j] = f of the j-th best matching row (best first, ties to the lowest
+ *   row id, the order of topk_select), out_idx[j] its row id; when fewer than k rows
+ *   match, rows j >= matches get out_idx = -1, out_keys = 0 bits, out_payload = 0.
+ *   Layout: every column (keys, rank_b, pred->col, payload) 16-byte aligned, same n;
+ *   1 <= k <= min(n, 1024); n <= 2^32 - 2.  Workspace: topk_workspace_bytes(dtype, n, k).
+ *   Errors: TOPK_ERR_INVALID_ARG for a misaligned column, a bad predicate kind, rank_b
+ *   with a non-F32 dtype, or neither pred nor rank_b (use topk_select). */
+typedef enum { TOPK_PRED_RANGE = 1, TOPK_PRED_IN = 2 } topk_pred_kind_t;
+typedef struct {
+    topk_pred_kind_t kind;
+    const uint32_t* col; /* DEVICE [n] */
+    uint32_t lo, hi;     /* TOPK_PRED_RANGE */
+    uint64_t in_mask;    /* TOPK_PRED_IN */
+} topk_pred_t;
+topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank_b,
+                         float rank_w, const topk_pred_t* pred, const uint32_t* payload,
+                         uint64_t n, uint32_t k, topk_order_t order, void* out_keys,
+                         uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
+                         void* stream);
+
 /* Top-k of keys in HOST memory (pinned memory strongly recommended): the input is
  * streamed to the device in chunks of `chunk_keys` keys through a double-buffered
  * staging area inside `ws`; each chunk's top-k runs as soon as it has landed, so the

@@ -7,6 +7,8 @@ C calls; every step of the top-k runs in the library's sm_100a kernels.
     values, indices = topk(x, k, largest=True)          # x: 1-D cuda f32/u32/f64
     values, indices, pay = topk(x, k, payload=p)        # key + 32-bit payload
     values, indices = merge(cand_vals, cand_idx, k)     # global step
+    values, indices = query(a, k, rank_b=b, rank_w=0.5, pred=("range", t, 0, X))
+                                                        # WHERE / ORDER BY f(A1, A2)
 """
 from __future__ import annotations
 
@@ -16,7 +18,7 @@ import torch
 
 from . import _lib
 
-__all__ = ["topk", "topk_host", "merge", "Workspace", "launch_count", "workspace_bytes"]
+__all__ = ["topk", "topk_host", "merge", "query", "Workspace", "launch_count", "workspace_bytes"]
 
 _DT = {torch.float32: _lib.F32, torch.uint32: _lib.U32, torch.float64: _lib.F64}
 
@@ -98,6 +100,58 @@ def topk(x: torch.Tensor, k: int, largest: bool = True, payload: torch.Tensor | 
                          _ptr(vals), _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
                          _stream_ptr(x.device))
     _lib.check(st, "topk_select")
+    return (vals, idx) if payload is None else (vals, idx, pay)
+
+
+def query(keys: torch.Tensor, k: int, largest: bool = True, rank_b: torch.Tensor | None = None,
+          rank_w: float = 0.0, pred: tuple | None = None, payload: torch.Tensor | None = None,
+          workspace: Workspace | None = None):
+    """``SELECT WHERE pred ORDER BY f DESC|ASC LIMIT k`` fused into one streaming pass
+    (the paper's §5: filter as the buffer filler, ranking function inside the pass).
+
+    ``pred``: ``("range", col, lo, hi)`` (lo <= col < hi) or ``("in", col, mask64)``
+    (col < 64 and bit col of mask); ``col`` a CUDA uint32 tensor.  ``rank_b``: None
+    (f = keys) or a CUDA float32 tensor (f = keys + rank_w * rank_b, f32, each op
+    rounded).  Every column 16-byte aligned.  Returns ``(values, indices)`` or
+    ``(values, indices, payload_out)``; rows beyond the matches have index -1.
+    """
+    if not keys.is_cuda or keys.dim() != 1:
+        raise ValueError("query expects 1-D CUDA tensors (no CPU path)")
+    lib = _lib.load()
+    dt = _dtype_code(keys)
+    n = keys.shape[0]
+    cols = [keys]
+    pr = None
+    if pred is not None:
+        if pred[0] == "range":
+            pr = _lib.Pred(_lib.PRED_RANGE, pred[1].data_ptr(), int(pred[2]), int(pred[3]), 0)
+        elif pred[0] == "in":
+            pr = _lib.Pred(_lib.PRED_IN, pred[1].data_ptr(), 0, 0, int(pred[2]))
+        else:
+            raise ValueError(f"unknown predicate kind {pred[0]!r}")
+        if pred[1].dtype != torch.uint32 or pred[1].shape[0] != n or not pred[1].is_contiguous():
+            raise ValueError("predicate column: contiguous CUDA uint32 of the same length")
+        cols.append(pred[1])
+    if rank_b is not None:
+        if rank_b.dtype != torch.float32 or rank_b.shape[0] != n or not rank_b.is_contiguous():
+            raise ValueError("rank_b: contiguous CUDA float32 of the same length")
+        cols.append(rank_b)
+    if payload is not None:
+        cols.append(payload)
+    if any(not c.is_contiguous() for c in cols):
+        raise ValueError("columns must be contiguous")
+    vals = torch.empty(k, dtype=keys.dtype, device=keys.device)
+    idx = torch.empty(k, dtype=torch.int64, device=keys.device)
+    pay = torch.empty(k, dtype=torch.uint32, device=keys.device) if payload is not None else None
+    need = int(lib.topk_workspace_bytes(dt, n, k))
+    if need == 0:
+        raise _lib.TopkError(f"invalid arguments for query (n={n}, k={k})")
+    ws = workspace if workspace is not None else _workspace(keys.device, need)
+    st = lib.topk_query(dt, _ptr(keys), _ptr(rank_b), float(rank_w),
+                        ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k,
+                        _lib.LARGEST if largest else _lib.SMALLEST, _ptr(vals), _ptr(pay),
+                        _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(keys.device))
+    _lib.check(st, "topk_query")
     return (vals, idx) if payload is None else (vals, idx, pay)
 
 

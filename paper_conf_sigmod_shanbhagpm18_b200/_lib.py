@@ -25,8 +25,15 @@ SYMBOLS = (
     "topk_launch_count", "topk_status_string", "topk_abi_version", "topk_probe_read",
     "topk_host_workspace_bytes", "topk_select_host", "topk_nccl_unique_id", "topk_nccl_comm_init",
     "topk_nccl_comm_destroy", "topk_sharded_workspace_bytes", "topk_select_sharded",
-    "topk_f32_sharded",
+    "topk_f32_sharded", "topk_query",
 )
+PRED_RANGE, PRED_IN = 1, 2
+
+
+class Pred(ctypes.Structure):
+    """topk_pred_t (include/topk.h)."""
+    _fields_ = [("kind", ctypes.c_int), ("col", ctypes.c_void_p), ("lo", ctypes.c_uint32),
+                ("hi", ctypes.c_uint32), ("in_mask", ctypes.c_uint64)]
 
 _lib = None
 
@@ -85,6 +92,9 @@ def load(build_if_missing: bool = True):
     lib.topk_select_sharded.restype = i32
     lib.topk_f32_sharded.argtypes = [vp, u64, u64, u32, i32, vp, vp, vp, vp, sz, vp]
     lib.topk_f32_sharded.restype = i32
+    lib.topk_query.argtypes = [i32, vp, vp, ctypes.c_float, ctypes.POINTER(Pred), vp, u64, u32,
+                               i32, vp, vp, vp, vp, sz, vp]
+    lib.topk_query.restype = i32
     lib.topk_launch_count.argtypes = []
     lib.topk_launch_count.restype = u64
     lib.topk_status_string.argtypes = [i32]

@@ -23,4 +23,14 @@ TOPK_DECLARE_SELECT_TU(u32)
 TOPK_DECLARE_SELECT_TU(f64)
 #undef TOPK_DECLARE_SELECT_TU
 
+// Query forms (select.cuh QCfg: q = kQPred | kQRank bits; kQRank for f32 only).
+#define TOPK_DECLARE_QUERY_TU(NAME)                                                         \
+    cudaError_t launch_query_##NAME(const SelectParams& p, int grid, bool min_order, int q, \
+                                    cudaStream_t st);                                       \
+    int debug_query_##NAME(int op, void* host, int arg);
+TOPK_DECLARE_QUERY_TU(f32)
+TOPK_DECLARE_QUERY_TU(u32)
+TOPK_DECLARE_QUERY_TU(f64)
+#undef TOPK_DECLARE_QUERY_TU
+
 }  // namespace topk

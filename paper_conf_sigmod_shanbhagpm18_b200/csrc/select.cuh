@@ -37,6 +37,8 @@
 #include "ptx.cuh"
 #include "wnet.cuh"
 
+#include <type_traits>
+
 namespace topk {
 
 #ifndef TOPK_VEC_PER_THREAD
@@ -71,6 +73,25 @@ struct Cfg {
     static_assert(kItems <= 32, "mask width");
 };
 
+// Query forms (the paper's §5 database integration; R17/R18): the
+// streamed row is more than the key column.  Q bits: kQPred -- a u32 predicate column
+// (WHERE), kQRank -- a second f32 column b with the ranking function f = a + w * b
+// (ORDER BY f).  A ring stage then holds one slab per column, TK rows each.
+constexpr int kQPred = 1, kQRank = 2;
+template <class Key, int Q>
+struct QCfg {
+    static constexpr int kRowBytes = static_cast<int>(sizeof(Key)) + ((Q & kQRank) ? 4 : 0) +
+                                     ((Q & kQPred) ? 4 : 0);
+    static constexpr int kItems =
+        Q == 0 ? Cfg<Key>::kItems : (kRowBytes <= 8 ? 8 : 4);  // rows per consumer thread
+    static constexpr int kTileKeys = Q == 0 ? Cfg<Key>::kTileKeys : kNC * kItems;
+    static constexpr int kVecPerThread = kItems / KeyTraits<Key>::kVec;
+    static constexpr int kOffB = kTileKeys * static_cast<int>(sizeof(Key));  // rank column b
+    static constexpr int kOffP = kOffB + ((Q & kQRank) ? kTileKeys * 4 : 0);  // predicate
+    static_assert(Q == 0 || kTileKeys * kRowBytes <= kTileBytes, "stage size");
+    static_assert(kTileKeys % 4 == 0, "TMA sizes are multiples of 16 bytes");
+};
+
 struct WsHeader {
     unsigned long long tau_g;  // max over CTAs of their k-th best
     unsigned int ticket;       // CTAs finished
@@ -100,7 +121,28 @@ struct SelectParams {
     uint32_t nwaves;   // ceil(nblocks / wave)
     uint32_t gmax;     // workspace layout: published-sample columns (>= gridDim.x)
     uint32_t J;        // published samples per CTA: the 2^j-th best of its run, j < J
+    // query forms (Q != 0; select_kernel's template argument)
+    const float* rank_b;   // kQRank: column b of f = key + rank_w * b
+    const uint32_t* pred;  // kQPred: predicate column
+    float rank_w;
+    uint32_t pred_in;      // 1: membership (pred < 64 and bit pred of pred_mask); 0: range
+    uint32_t pred_lo;      // range: pred_lo <= pred < pred_lo + pred_span
+    uint32_t pred_span;
+    uint64_t pred_mask;
 };
+
+// WHERE (reading R17): range lo <= v < lo + span as one unsigned compare, or IN-list
+// membership over dictionary codes < 64.
+__device__ __forceinline__ bool pred_ok(const SelectParams& p, uint32_t v) {
+    const bool in = v < 64u && ((p.pred_mask >> (v & 63u)) & 1ull);
+    const bool rg = v - p.pred_lo < p.pred_span;
+    return p.pred_in ? in : rg;
+}
+// ORDER BY f (reading R18): f = a + w * b, the product and the sum each rounded to
+// nearest f32 (no fused multiply-add, so the oracle's plain C arithmetic agrees).
+__device__ __forceinline__ float rank_f(float a, float w, float b) {
+    return __fadd_rn(a, __fmul_rn(w, b));
+}
 
 // Workspace: [WsHeader | pub: u64[kPubRows][gmax] | cand: G x k entries]
 __host__ __device__ constexpr size_t ws_pub_offset() { return 64; }
@@ -734,13 +776,132 @@ __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
     return old;
 }
 
-template <class Key, bool MIN, bool FILTER>
+// Query form of consume_tile (Q != 0; filter mode): the row's key is the key column
+// (or f = a + w * b), and a row enters the buffer filler only if it satisfies the
+// predicate -- "apply the filter predicate ... and then [write] it out into a shared
+// memory buffer" (FusedSortReducer), with the top-k bound as a second predicate.
+// Keys stay in registers (<= 8 per thread) for the exact test.
+template <class Key, bool MIN, int Q>
+__device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
+                                              const Par<typename KeyTraits<Key>::E, Key>& pr,
+                                              uint32_t tlen, uint32_t lbase,
+                                              const SBuf<typename KeyTraits<Key>::E>& buf,
+                                              int* s_cnt, int limit, const SelectParams& p) {
+    using KT = KeyTraits<Key>;
+    using E = typename KT::E;
+    using Vec = typename KT::Vec;
+    using QC = QCfg<Key, Q>;
+    constexpr int VEC = KT::kVec;
+    constexpr int VPT = QC::kVecPerThread;
+    constexpr int ITEMS = QC::kItems;
+    constexpr int TK = QC::kTileKeys;
+    // 4-byte secondary columns, VEC lanes at the key vector's positions
+    using UVec = typename std::conditional<VEC == 4, uint4, uint2>::type;
+    const int tid = threadIdx.x;
+    const int lane = tid & 31;
+
+    Key x[ITEMS];
+    {
+        const Vec* sv = reinterpret_cast<const Vec*>(slot_data);
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const Vec v = sv[tid + j * kNC];
+#pragma unroll
+            for (int w = 0; w < VEC; ++w) x[j * VEC + w] = vget(v, w);
+        }
+    }
+    if constexpr ((Q & kQRank) != 0) {
+        static_assert(sizeof(Key) == 4 && VEC == 4, "ranking function: f32 columns");
+        const float4* sb = reinterpret_cast<const float4*>(slot_data + QC::kOffB);
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const float4 b = sb[tid + j * kNC];
+#pragma unroll
+            for (int w = 0; w < VEC; ++w) x[j * VEC + w] = rank_f(x[j * VEC + w], p.rank_w, vget(b, w));
+        }
+    }
+    uint32_t pm = (ITEMS >= 32) ? 0xFFFFFFFFu : ((1u << ITEMS) - 1u);
+    if constexpr ((Q & kQPred) != 0) {
+        const UVec* sp = reinterpret_cast<const UVec*>(slot_data + QC::kOffP);
+        pm = 0;
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const UVec u = sp[tid + j * kNC];
+#pragma unroll
+            for (int w = 0; w < VEC; ++w)
+                pm |= static_cast<uint32_t>(pred_ok(p, vget(u, w))) << (j * VEC + w);
+        }
+    }
+    auto pos_of = [&](int q) -> uint32_t {
+        return static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
+    };
+    if (tlen < static_cast<uint32_t>(TK)) {
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q)
+            if (pos_of(q) >= tlen) pm &= ~(1u << q);
+    }
+    uint32_t mask = pm;
+    if (pr.active) {
+        const bool strict = lbase > pr.strict_after;
+        uint32_t f = 0;
+        if (strict) {
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                f |= static_cast<uint32_t>(KT::template fast<MIN, true>(x[q], pr.t)) << q;
+        } else {
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                f |= static_cast<uint32_t>(KT::template fast<MIN, false>(x[q], pr.t)) << q;
+        }
+        mask &= f;
+    }
+    if (!__any_sync(0xFFFFFFFFu, mask != 0u)) return 0;
+    uint32_t keep = mask;
+    if (pr.active) {  // exact entry test (R1 order) on the passing rows
+        keep = 0;
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q)
+            if (((mask >> q) & 1u) &&
+                better(E::make(KT::template code<MIN>(x[q]), lbase + pos_of(q)), pr.tau))
+                keep |= 1u << q;
+    }
+    const int cnt = __popc(keep);
+    int incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
+        if (lane >= o) incl += y;
+    }
+    const int total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+    if (total == 0) return 0;
+    int old = 0;
+    if (lane == 31) old = reserve(s_cnt, total, limit);
+    old = __shfl_sync(0xFFFFFFFFu, old, 31);
+    if (old < 0) return -1;
+    int w = old + incl - cnt;
+#pragma unroll
+    for (int q = 0; q < ITEMS; ++q)
+        if ((keep >> q) & 1u) buf.st(w++, E::make(KT::template code<MIN>(x[q]), lbase + pos_of(q)));
+    return old;
+}
+
+// The key of global row `row` under query form Q (the extras and the finalize gather).
+template <class Key, int Q>
+__device__ __forceinline__ Key query_key(const SelectParams& p, const Key* keys, uint64_t row) {
+    if constexpr ((Q & kQRank) != 0)
+        return rank_f(keys[row], p.rank_w, p.rank_b[row]);
+    else
+        return keys[row];
+}
+
+template <class Key, bool MIN, bool FILTER, int Q = 0>
 __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     using KT = KeyTraits<Key>;
     using E = typename KT::E;
     using C = Cfg<Key>;
-    constexpr int TK = C::kTileKeys;
+    constexpr int TK = QCfg<Key, Q>::kTileKeys;
     constexpr int kStages = C::kStages;
+    static_assert(Q == 0 || FILTER, "query forms run in filter mode");
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ CtaState<E, Key> st;
@@ -802,12 +963,24 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     if (c == 0) {
         const uint64_t tail0 = p.head + p.body_n;
         const int nextra = static_cast<int>(p.head + (p.n - tail0));
-        if (tid < nextra) {
-            const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
-                                                                 : tail0 + (tid - p.head);
-            buf.st(tid, E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row)));
+        if constexpr (Q == 0) {
+            if (tid < nextra) {
+                const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
+                                                                     : tail0 + (tid - p.head);
+                buf.st(tid, E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row)));
+            }
+            if (tid == 0) st.cnt = nextra;
+        } else if (tid < 32) {  // query forms: head == 0, nextra <= 3; WHERE applies
+            const uint64_t row = tail0 + tid;
+            bool ok = tid < nextra;
+            if constexpr ((Q & kQPred) != 0) ok = ok && pred_ok(p, p.pred[ok ? row : 0]);
+            const uint32_t bal = __ballot_sync(0xFFFFFFFFu, ok);
+            if (ok)
+                buf.st(__popc(bal & ((1u << tid) - 1u)),
+                       E::make(KT::template code<MIN>(query_key<Key, Q>(p, keys, row)),
+                               static_cast<uint32_t>(row)));
+            if (tid == 0) st.cnt = __popc(bal);
         }
-        if (tid == 0) st.cnt = nextra;
     }
     __syncthreads();
 
@@ -853,9 +1026,19 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             }
             const uint64_t lo = static_cast<uint64_t>(tile) * TK;
             const uint64_t len = min(static_cast<uint64_t>(TK), p.body_n - lo);
-            const uint32_t bytes = static_cast<uint32_t>(len * sizeof(Key));
-            tma_load_1d(ring + static_cast<size_t>(slot) * kTileBytes, body + lo, bytes, &full[slot],
-                        policy);
+            uint32_t bytes = static_cast<uint32_t>(len * sizeof(Key));
+            unsigned char* dst = ring + static_cast<size_t>(slot) * kTileBytes;
+            tma_load_1d(dst, body + lo, bytes, &full[slot], policy);
+            if constexpr ((Q & kQRank) != 0) {  // one slab per column (query forms: head == 0)
+                tma_load_1d(dst + QCfg<Key, Q>::kOffB, p.rank_b + lo,
+                            static_cast<uint32_t>(len * 4), &full[slot], policy);
+                bytes += static_cast<uint32_t>(len * 4);
+            }
+            if constexpr ((Q & kQPred) != 0) {
+                tma_load_1d(dst + QCfg<Key, Q>::kOffP, p.pred + lo, static_cast<uint32_t>(len * 4),
+                            &full[slot], policy);
+                bytes += static_cast<uint32_t>(len * 4);
+            }
             mbar_arrive_expect_tx(&full[slot], bytes);  // release: tile id visible
         }
     }
@@ -892,7 +1075,13 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         const uint32_t lbase = static_cast<uint32_t>(p.head + tlo);
         const unsigned char* data = ring + static_cast<size_t>(slot) * kTileBytes;
         Par<E, Key> pr = load_par<Key, MIN>(st);
-        int r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, st.limit);
+        auto consume = [&]() -> int {
+            if constexpr (Q == 0)
+                return consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, st.limit);
+            else
+                return consume_tile_q<Key, MIN, Q>(data, pr, tlen, lbase, buf, &st.cnt, st.limit, p);
+        };
+        int r = consume();
         while (r < 0) {  // did not fit: flush, then redo with the new bound
             if (lane == 0) {
                 atomicAdd(&g_stats[3], 1ull);
@@ -902,7 +1091,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             cbar_or(true);
             collective();
             pr = load_par<Key, MIN>(st);
-            r = consume_tile<Key, MIN, FILTER>(data, pr, tlen, lbase, buf, &st.cnt, st.limit);
+            r = consume();
         }
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[slot]);
@@ -1063,14 +1252,16 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     // ---- finalize: best first, original key bits, global index, payload ----
     for (int j = tid; j < k; j += kNC) {
         const E e = buf.ld(j);
-        if (e.is_sentinel()) {  // cannot happen (k <= n); never read out of bounds
-            atomicAdd(&g_stats[7], 1ull);
+        if (e.is_sentinel()) {  // fewer than k rows (only a WHERE can do that, since k <= n)
+            if (Q == 0) atomicAdd(&g_stats[7], 1ull);  // plain form: a bug
             if (p.out_idx) p.out_idx[j] = -1;
+            if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = Key(0);
+            if (p.out_payload) p.out_payload[j] = 0u;
             continue;
         }
         const uint32_t row = e.lidx();
         if (p.out_idx) p.out_idx[j] = static_cast<int64_t>(p.base + row);
-        if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = keys[row];
+        if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = query_key<Key, Q>(p, keys, row);
         if (p.out_payload) p.out_payload[j] = p.payload[row];
     }
     if (tid == 0) trace(6);

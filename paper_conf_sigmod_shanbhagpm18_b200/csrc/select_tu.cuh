@@ -1,6 +1,9 @@
 // select_tu.cuh -- body of one select translation unit: instantiates select_kernel for
 // one key type (both orders, filter and pure modes) and the TU's debug accessors.
 // Include after defining TOPK_TU_KEY (the key type) and TOPK_TU_NAME (f32 | u32 | f64).
+// With TOPK_TU_QUERY defined the TU instead instantiates the query forms (WHERE
+// predicate; for f32 also the ranking function), as launch_query_<NAME> /
+// debug_query_<NAME>.
 #pragma once
 #include <atomic>
 
@@ -13,23 +16,25 @@
 namespace topk {
 namespace {
 
-template <class Key, bool MIN, bool FILTER>
+template <class Key, bool MIN, bool FILTER, int Q = 0>
 cudaError_t launch_one(const SelectParams& p, int grid, cudaStream_t st) {
     static std::atomic<bool> attr_set{false};  // per instantiation (idempotent)
     const size_t smem = select_smem_bytes<Key>();
     if (!attr_set.load(std::memory_order_relaxed)) {
-        cudaError_t e = cudaFuncSetAttribute(select_kernel<Key, MIN, FILTER>,
+        cudaError_t e = cudaFuncSetAttribute(select_kernel<Key, MIN, FILTER, Q>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              static_cast<int>(smem));
         if (e != cudaSuccess) return e;
         attr_set.store(true, std::memory_order_relaxed);
     }
-    select_kernel<Key, MIN, FILTER><<<grid, kNT, smem, st>>>(p);
+    select_kernel<Key, MIN, FILTER, Q><<<grid, kNT, smem, st>>>(p);
     return cudaGetLastError();
 }
 
 }  // namespace
 
+#ifndef TOPK_TU_QUERY
+#define TOPK_TU_KIND select_
 cudaError_t TOPK_CAT(launch_select_, TOPK_TU_NAME)(const SelectParams& p, int grid,
                                                    bool min_order, bool filter,
                                                    cudaStream_t st) {
@@ -40,8 +45,33 @@ cudaError_t TOPK_CAT(launch_select_, TOPK_TU_NAME)(const SelectParams& p, int gr
     return filter ? launch_one<Key, false, true>(p, grid, st)
                   : launch_one<Key, false, false>(p, grid, st);
 }
+#else
+#define TOPK_TU_KIND query_
+cudaError_t TOPK_CAT(launch_query_, TOPK_TU_NAME)(const SelectParams& p, int grid,
+                                                  bool min_order, int q, cudaStream_t st) {
+    using Key = TOPK_TU_KEY;
+    if constexpr (sizeof(Key) == 4 && static_cast<Key>(-1) < static_cast<Key>(0)) {  // f32
+        switch (q) {
+            case kQPred:
+                return min_order ? launch_one<Key, true, true, kQPred>(p, grid, st)
+                                 : launch_one<Key, false, true, kQPred>(p, grid, st);
+            case kQRank:
+                return min_order ? launch_one<Key, true, true, kQRank>(p, grid, st)
+                                 : launch_one<Key, false, true, kQRank>(p, grid, st);
+            case kQPred | kQRank:
+                return min_order ? launch_one<Key, true, true, kQPred | kQRank>(p, grid, st)
+                                 : launch_one<Key, false, true, kQPred | kQRank>(p, grid, st);
+        }
+        return cudaErrorInvalidValue;
+    } else {
+        if (q != kQPred) return cudaErrorInvalidValue;
+        return min_order ? launch_one<Key, true, true, kQPred>(p, grid, st)
+                         : launch_one<Key, false, true, kQPred>(p, grid, st);
+    }
+}
+#endif
 
-int TOPK_CAT(debug_select_, TOPK_TU_NAME)(int op, void* host, int arg) {
+int TOPK_CAT(TOPK_CAT(debug_, TOPK_TU_KIND), TOPK_TU_NAME)(int op, void* host, int arg) {
     switch (op) {
         case kDbgStatsAdd: {  // host: u64[8], accumulated
             unsigned long long v[8];

@@ -73,9 +73,22 @@ cudaError_t dispatch_select(topk_dtype_t dt, const topk::SelectParams& p, int gr
     return e;
 }
 
+cudaError_t dispatch_query(topk_dtype_t dt, const topk::SelectParams& p, int grid,
+                           bool min_order, int q, cudaStream_t st) {
+    cudaError_t e;
+    switch (dt) {
+        case TOPK_F32: e = topk::launch_query_f32(p, grid, min_order, q, st); break;
+        case TOPK_U32: e = topk::launch_query_u32(p, grid, min_order, q, st); break;
+        default: e = topk::launch_query_f64(p, grid, min_order, q, st); break;
+    }
+    if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
+    return e;
+}
+
 // Every select translation unit's debug accessor (each holds its own device globals).
 int (*const kSelectDebug[])(int, void*, int) = {topk::debug_select_f32, topk::debug_select_u32,
-                                                topk::debug_select_f64};
+                                                topk::debug_select_f64, topk::debug_query_f32,
+                                                topk::debug_query_u32, topk::debug_query_f64};
 
 template <class Key, bool MIN>
 cudaError_t launch_merge(const topk::MergeParams& p, cudaStream_t st) {
@@ -107,6 +120,19 @@ uint32_t tile_keys_for(topk_dtype_t dt) {
         case TOPK_F64: return tile_keys<double>();
         case TOPK_U32: return tile_keys<uint32_t>();
         default: return tile_keys<float>();
+    }
+}
+
+uint32_t query_tile_keys(topk_dtype_t dt, int q) {
+    using topk::QCfg;
+    using topk::kQPred;
+    using topk::kQRank;
+    if (dt == TOPK_F64) return QCfg<double, kQPred>::kTileKeys;
+    if (dt == TOPK_U32) return QCfg<uint32_t, kQPred>::kTileKeys;
+    switch (q) {
+        case kQRank: return QCfg<float, kQRank>::kTileKeys;
+        case kQRank | kQPred: return QCfg<float, kQRank | kQPred>::kTileKeys;
+        default: return QCfg<float, kQPred>::kTileKeys;
     }
 }
 
@@ -166,10 +192,19 @@ topk_status_t topk_workspace_init(void* ws, size_t ws_bytes, void* stream) {
     return TOPK_OK;
 }
 
+// Query forms (topk_query): q = kQPred | kQRank bits, 0 for a plain top-k.
+struct QueryArgs {
+    int q = 0;
+    const float* rank_b = nullptr;
+    float rank_w = 0.f;
+    topk_pred_t pred{};
+};
+
 static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
                           uint64_t n, uint64_t base, uint32_t k, topk_order_t order,
                           topk_mode_t mode, void* out_keys, uint32_t* out_payload,
-                          int64_t* out_idx, void* ws, size_t ws_bytes, void* stream) {
+                          int64_t* out_idx, void* ws, size_t ws_bytes, void* stream,
+                          const QueryArgs& qa = QueryArgs()) {
     if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
     if (mode != TOPK_MODE_FILTER && mode != TOPK_MODE_PURE) return TOPK_ERR_INVALID_ARG;
     if (!keys || n == 0 || k == 0 || k > TOPK_MAX_K || k > n) return TOPK_ERR_INVALID_ARG;
@@ -196,9 +231,22 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
     const uint64_t vec = 16 / ks;
     uint64_t head = ((16 - (addr % 16)) % 16) / ks;
     if (head > n) head = n;
+    if (qa.q) head = 0;  // topk_query: 16-byte aligned columns
     p.head = static_cast<uint32_t>(head);
-    p.body_n = (n - head) / vec * vec;
-    const uint32_t tk = tile_keys_for(dtype);
+    // query forms: the 4-byte columns' slabs need multiples of 4 rows (16 B) per copy
+    p.body_n = qa.q ? n / 4 * 4 : (n - head) / vec * vec;
+    const uint32_t tk = qa.q ? query_tile_keys(dtype, qa.q) : tile_keys_for(dtype);
+    if (qa.q) {
+        p.rank_b = qa.rank_b;
+        p.rank_w = qa.rank_w;
+        if (qa.q & topk::kQPred) {
+            p.pred = qa.pred.col;
+            p.pred_in = qa.pred.kind == TOPK_PRED_IN ? 1u : 0u;
+            p.pred_lo = qa.pred.lo;
+            p.pred_span = qa.pred.hi > qa.pred.lo ? qa.pred.hi - qa.pred.lo : 0u;
+            p.pred_mask = qa.pred.in_mask;
+        }
+    }
     const uint64_t ntiles = (p.body_n + tk - 1) / tk;
     p.ntiles = static_cast<uint32_t>(ntiles);
     p.k = k;
@@ -236,6 +284,7 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
+    if (qa.q) return dispatch_query(dtype, p, grid, mn, qa.q, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
     return dispatch_select(dtype, p, grid, mn, filt, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
 }
 
@@ -275,6 +324,34 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
     return merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
                        payload ? reinterpret_cast<const uint32_t*>(w + L.cp) : nullptr, total, k,
                        order, out_keys, out_payload, out_idx, stream);
+}
+
+topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank_b,
+                         float rank_w, const topk_pred_t* pred, const uint32_t* payload,
+                         uint64_t n, uint32_t k, topk_order_t order, void* out_keys,
+                         uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
+                         void* stream) {
+    if (!valid_dtype(dtype) || !keys || n == 0 || n > kMaxLaunchN) return TOPK_ERR_INVALID_ARG;
+    QueryArgs qa;
+    if (rank_b) {
+        if (dtype != TOPK_F32) return TOPK_ERR_INVALID_ARG;
+        qa.q |= topk::kQRank;
+        qa.rank_b = rank_b;
+        qa.rank_w = rank_w;
+    }
+    if (pred) {
+        if ((pred->kind != TOPK_PRED_RANGE && pred->kind != TOPK_PRED_IN) || !pred->col)
+            return TOPK_ERR_INVALID_ARG;
+        qa.q |= topk::kQPred;
+        qa.pred = *pred;
+    }
+    if (!qa.q) return TOPK_ERR_INVALID_ARG;
+    auto misaligned = [](const void* c) { return reinterpret_cast<uintptr_t>(c) % 16 != 0; };
+    if (misaligned(keys) || (rank_b && misaligned(rank_b)) || (pred && misaligned(pred->col)) ||
+        (payload && misaligned(payload)))
+        return TOPK_ERR_INVALID_ARG;
+    return select_one(dtype, keys, payload, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                      out_payload, out_idx, ws, ws_bytes, stream, qa);
 }
 
 topk_status_t topk_f32(const float* keys, uint64_t n, uint32_t k, topk_order_t order,

@@ -1,0 +1,154 @@
+"""GPU parity of the query form (topk_query: WHERE predicate fused as the buffer
+filler, ORDER BY a ranking function evaluated inside the pass -- the paper's §5,
+P:216-224) against the oracle's unfused plan (filter, project, top-k), bit-exact in
+values and indices.  Inputs from the shared seeded generator; expected values only
+from oracle/."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_sigmod_shanbhagpm18_b200 as tk
+from paper_conf_sigmod_shanbhagpm18_b200 import _lib, datagen
+
+pytestmark = pytest.mark.gpu
+
+
+def host(t: torch.Tensor) -> np.ndarray:
+    if t.dtype == torch.uint32:
+        return t.cpu().view(torch.int32).numpy().view(np.uint32)
+    return t.cpu().numpy()
+
+
+def u32col(n, seed, mod=None):
+    c = datagen.generate("uniform", n, "u32", seed=seed)
+    if mod is not None:
+        c = (c.to(torch.int64) % mod).to(torch.uint32)
+    return c
+
+
+def run(keys, k, largest=True, rank_b=None, w=0.0, pred=None, payload=None):
+    """GPU query vs oracle.query on the same host columns."""
+    dev = "cuda"
+    gpred = None if pred is None else (pred[0], pred[1].to(dev), *pred[2:])
+    out = tk.query(keys.to(dev), k, largest, rank_b=None if rank_b is None else rank_b.to(dev),
+                   rank_w=w, pred=gpred, payload=None if payload is None else payload.to(dev))
+    torch.cuda.synchronize()
+    hpred = None if pred is None else (pred[0], host(pred[1]), *pred[2:])
+    ov, oi, m = oracle.query(host(keys), k, largest,
+                             rank_b=None if rank_b is None else host(rank_b), rank_w=w,
+                             pred=hpred)
+    gi = out[1].cpu().numpy()
+    assert np.array_equal(gi, oi), f"indices differ (m={m}): first at {np.nonzero(gi != oi)[0][:5]}"
+    assert host(out[0]).tobytes() == ov.tobytes(), "value bits differ"
+    if payload is not None:
+        ph = host(payload)
+        exp = np.where(oi >= 0, ph[np.maximum(oi, 0)], 0).astype(np.uint32)
+        assert np.array_equal(host(out[2]), exp)
+    return m
+
+
+N = (1 << 20) + 4096 * 3 + 7  # many tiles, ragged tail (n % 4 != 0)
+
+
+@pytest.mark.parametrize("dt", ["f32", "u32", "f64"])
+@pytest.mark.parametrize("largest", [True, False])
+def test_range_predicate_selectivities(cuda_device, dt, largest):
+    keys = datagen.generate("uniform", N, dt, seed=301)
+    col = u32col(N, 302, 1000)
+    for lo, hi in [(0, 1000), (0, 500), (250, 260), (999, 1000), (0, 0)]:
+        for k in (1, 50, 256):
+            run(keys, k, largest, pred=("range", col, lo, hi))
+
+
+@pytest.mark.parametrize("k", [1, 7, 32, 64, 100, 256, 512, 1024])
+def test_every_k_in_predicate(cuda_device, k):
+    keys = datagen.generate("uniform", N, "f32", seed=303)
+    lang = u32col(N, 304, 70)  # dictionary codes; >= 64 never match
+    run(keys, k, True, pred=("in", lang, (1 << 3) | (1 << 5)))
+    run(keys, k, False, pred=("in", lang, 1 << 63))
+
+
+@pytest.mark.parametrize("largest", [True, False])
+def test_ranking_function(cuda_device, largest):
+    a = datagen.generate("uniform", N, "f32", seed=305)
+    b = datagen.generate("uniform", N, "f32", seed=306)
+    for w in (0.5, -1.25, 3.0e-3):
+        for k in (1, 64, 256, 1000):
+            run(a, k, largest, rank_b=b, w=w)
+
+
+def test_ranking_special_values(cuda_device):
+    a = datagen.generate("uniform", 100000, "f32", seed=307)
+    b = datagen.generate("uniform", 100000, "f32", seed=308)
+    sp_a = torch.tensor([float("nan"), -0.0, 0.0, float("inf"), -float("inf"), 1e-40, 2.0, 1.0],
+                        dtype=torch.float32)
+    sp_b = torch.tensor([1.0, 0.0, -0.0, -1.0, 5.0, 1e-40, float("nan"), float("inf")],
+                        dtype=torch.float32)
+    for j in range(8):
+        a[j * 9973] = sp_a[j]
+        b[j * 9973] = sp_b[j]
+    for largest in (True, False):
+        run(a, 20, largest, rank_b=b, w=0.5)
+
+
+def test_integer_counts_query2(cuda_device):
+    """P:298 query 2: retweet_count + 0.5 * likes_count (integer counts in f32)."""
+    rt = (u32col(N, 309, 5000).to(torch.float32))
+    likes = (u32col(N, 310, 20000).to(torch.float32))
+    run(rt, 50, True, rank_b=likes, w=0.5)
+
+
+def test_rank_and_predicate(cuda_device):
+    a = datagen.generate("uniform", N, "f32", seed=311)
+    b = datagen.generate("uniform", N, "f32", seed=312)
+    t = u32col(N, 313)
+    run(a, 256, True, rank_b=b, w=0.5, pred=("range", t, 0, 1 << 30))
+    run(a, 64, False, rank_b=b, w=2.0, pred=("in", (t.to(torch.int64) % 64).to(torch.uint32), 0xF0F0))
+
+
+def test_fewer_matches_than_k(cuda_device):
+    keys = datagen.generate("uniform", N, "f32", seed=314)
+    rowid = torch.arange(N, dtype=torch.int64).to(torch.uint32)
+    for lo, hi in [(5, 5), (100, 120), (N - 3, N), (N - 1000, N)]:
+        m = run(keys, 256, True, pred=("range", rowid, lo, hi))
+        assert m == min(256, hi - lo)
+
+
+@pytest.mark.parametrize("dist", ["increasing", "decreasing", "fewdistinct"])
+def test_adversarial_with_time_predicate(cuda_device, dist):
+    """Query 1 shape: WHERE tweet_time < X, time = row order (appended log)."""
+    keys = datagen.generate(dist, N, "f32", seed=315)
+    t = torch.arange(N, dtype=torch.int64).to(torch.uint32)
+    for X in (N // 10, N // 2, N):
+        run(keys, 50, True, pred=("range", t, 0, X))
+        run(keys, 50, False, pred=("range", t, 0, X))
+
+
+def test_payload_and_small_n(cuda_device):
+    for n in (1, 3, 4, 5, 17, 4096, 7681):
+        keys = datagen.generate("uniform", n, "f32", seed=316 + n)
+        col = u32col(n, 317, 4)
+        pay = datagen.payload(n, seed=318)
+        k = min(n, 16)
+        run(keys, k, True, pred=("range", col, 1, 3), payload=pay)
+
+
+def test_rejects_bad_arguments(cuda_device):
+    keys = torch.rand(1024, device="cuda")
+    col = torch.zeros(1024, dtype=torch.uint32, device="cuda")
+    with pytest.raises(_lib.TopkError):  # misaligned column
+        tk.query(keys[1:], 8, pred=("range", col[1:], 0, 1))
+    with pytest.raises(_lib.TopkError):  # ranking function needs f32
+        tk.query(keys.double(), 8, rank_b=keys)
+    with pytest.raises(_lib.TopkError):  # neither predicate nor ranking function
+        tk.query(keys, 8)
+
+
+@pytest.mark.slow
+def test_full_size_query1(cuda_device):
+    """2^28 rows (BJ config-4 size): WHERE time < X ORDER BY count DESC LIMIT 50."""
+    n = 1 << 28
+    keys = datagen.generate("uniform", n, "u32", seed=319)
+    t = u32col(n, 320)
+    run(keys, 50, True, pred=("range", t, 0, 1 << 31))
