@@ -286,6 +286,28 @@ def run_ours(args):
         cfgs.append({"config": "BJ4b: 2^28 f64, DESC LIMIT 64", "us": round(t * 1e3, 1),
                      "keys_per_s": n4 / (t / 1e3), "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
         del xd64
+        # f1: the paper's §5 query forms fused into the pass (queries 1-3 of
+        # §6.8): 2^28 rows, 8 bytes streamed per row (key column + one more column)
+        cnt = datagen.generate("uniform", n4, "u32", seed=datagen.config_seed(6), device=dev)
+        tcol = datagen.generate("uniform", n4, "u32", seed=datagen.config_seed(6, 1), device=dev)
+        lang = (tcol.view(torch.int32) & 63).view(torch.uint32)  # dictionary codes 0..63
+        for name, fq in (
+                ("query1: WHERE time < 2^31 (sel 0.5) ORDER BY count DESC LIMIT 50 (u32 cols)",
+                 lambda: tk.query(cnt, 50, True, pred=("range", tcol, 0, 1 << 31))),
+                ("query3: WHERE lang IN (52 of 64 codes, sel 0.81) ORDER BY count DESC LIMIT 50",
+                 lambda: tk.query(cnt, 50, True, pred=("in", lang, (1 << 52) - 1)))):
+            t = timed(fq)
+            cfgs.append({"config": f"f1 {name}", "us": round(t * 1e3, 1),
+                         "rows_per_s": n4 / (t / 1e3),
+                         "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
+        del cnt, tcol, lang
+        a = datagen.generate("uniform", n4, "f32", seed=datagen.config_seed(6, 2), device=dev)
+        b = datagen.generate("uniform", n4, "f32", seed=datagen.config_seed(6, 3), device=dev)
+        t = timed(lambda: tk.query(a, 50, True, rank_b=b, rank_w=0.5))
+        cfgs.append({"config": "f1 query2: ORDER BY a + 0.5 * b DESC LIMIT 50 (f32 cols)",
+                     "us": round(t * 1e3, 1), "rows_per_s": n4 / (t / 1e3),
+                     "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
+        del a, b
         for kk in (32, 256):
             t = timed(lambda: tk.topk(x, kk, True, mode="pure"), 2)
             cfgs.append({"config": f"pure mode (paper's data-independent network on every key), "

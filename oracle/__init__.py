@@ -54,6 +54,8 @@ def _load():
         lib.oracle_query.argtypes = [i32, vp, vp, ctypes.c_float, i32, vp, u32, u32, u64, u64,
                                      u32, i32, vp, vp, i32]
         lib.oracle_query.restype = i32
+        lib.oracle_topk_kk.argtypes = [vp, vp, u64, u32, i32, i32, vp, vp, vp]
+        lib.oracle_topk_kk.restype = i32
         lib.oracle_threads.argtypes = []
         lib.oracle_threads.restype = i32
         _lib = lib
@@ -123,6 +125,24 @@ def query(keys: np.ndarray, k: int, largest: bool = True, rank_b: np.ndarray | N
     if m < 0:
         raise ValueError("oracle_query: invalid arguments")
     return out_k, out_i, m
+
+
+def topk_kk(k1: np.ndarray, k2: np.ndarray, k: int, largest1: bool = True,
+            largest2: bool = True):
+    """Compound-key top-k (ORDER BY k1, k2 LIMIT k; KKV): lexicographic on
+    the two float32 columns' order codes, then the lowest row id.  Returns
+    ``(v1, v2, indices)``."""
+    k1 = np.ascontiguousarray(k1, dtype=np.float32)
+    k2 = np.ascontiguousarray(k2, dtype=np.float32)
+    assert k1.shape == k2.shape
+    o1 = np.empty(k, dtype=np.float32)
+    o2 = np.empty(k, dtype=np.float32)
+    oi = np.empty(k, dtype=np.int64)
+    r = _load().oracle_topk_kk(_ptr(k1), _ptr(k2), k1.shape[0], k, 0 if largest1 else 1,
+                               0 if largest2 else 1, _ptr(o1), _ptr(o2), _ptr(oi))
+    if r < 0:
+        raise ValueError("oracle_topk_kk: invalid arguments")
+    return o1, o2, oi
 
 
 def certificate(keys: np.ndarray, k: int, out_keys: np.ndarray, out_idx: np.ndarray,

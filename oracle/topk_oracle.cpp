@@ -256,6 +256,41 @@ int oracle_query(int dtype, const void* keys, const float* rank_b, float w, int 
     return static_cast<int>(kk);
 }
 
+/* Compound keys (§6.6 "two keys + value (KKV)"; reading R19):
+ *   ORDER BY k1 [DESC|ASC], k2 [DESC|ASC] LIMIT k  over two f32 columns
+ * -- lexicographic: k1 decides, k2 breaks k1 ties, then the lowest row id.  Each
+ * column's order is that of oracle_topk's code map (order1 / order2).  The compare is
+ * written as the plain lexicographic rule on the two codes (no packing), and the
+ * value (payload) is the tuple id gathered at the end.  Writes out_k1[k],
+ * out_k2[k] (original bits), out_idx[k]; returns 0 or -1 on an argument error. */
+int oracle_topk_kk(const float* k1, const float* k2, uint64_t n, uint32_t k, int order1,
+                   int order2, float* out_k1, float* out_k2, int64_t* out_idx) {
+    if (!k1 || !k2 || n == 0 || k == 0 || k > n) return -1;
+    if ((order1 != 0 && order1 != 1) || (order2 != 0 && order2 != 1)) return -1;
+    struct Row {
+        uint64_t c1, c2, idx;
+    };
+    std::vector<Row> v(n);
+    for (uint64_t i = 0; i < n; ++i) {
+        v[i].c1 = code_of(DT_F32, k1, i, order1);
+        v[i].c2 = code_of(DT_F32, k2, i, order2);
+        v[i].idx = i;
+    }
+    auto lex_better = [](const Row& a, const Row& b) {
+        if (a.c1 != b.c1) return a.c1 > b.c1;
+        if (a.c2 != b.c2) return a.c2 > b.c2;
+        return a.idx < b.idx;
+    };
+    std::partial_sort(v.begin(), v.begin() + k, v.end(), lex_better);
+    for (uint32_t j = 0; j < k; ++j) {
+        const uint64_t r = v[j].idx;
+        if (out_idx) out_idx[j] = static_cast<int64_t>(r);
+        if (out_k1) std::memcpy(out_k1 + j, k1 + r, 4);
+        if (out_k2) std::memcpy(out_k2 + j, k2 + r, 4);
+    }
+    return 0;
+}
+
 /* Order code of each key (exposed so tests can pin the code map itself against
  * IEEE-754 facts and against library sorts). */
 void oracle_codes(int dtype, const void* keys, uint64_t n, int order, uint64_t* out) {

@@ -132,3 +132,73 @@ def test_closed_forms():
     v, i, m = oracle.query(a, 64, True, rank_b=b, rank_w=0.0)
     sv, si = oracle.topk(a, 64, True)
     assert np.array_equal(i, si) and v.tobytes() == sv.tobytes()
+
+
+# ---- compound keys (KKV; R19) ----
+
+def lex_ref(k1, k2, k, l1, l2):
+    """numpy.lexsort (last key primary) on NaN-free columns: the library pin."""
+    s1 = -k1.astype(np.float64) if l1 else k1.astype(np.float64)
+    s2 = -k2.astype(np.float64) if l2 else k2.astype(np.float64)
+    order = np.lexsort((np.arange(k1.shape[0]), s2, s1))[:k]
+    return order
+
+
+@pytest.mark.parametrize("l1", [True, False])
+@pytest.mark.parametrize("l2", [True, False])
+def test_compound_keys_vs_lexsort(l1, l2):
+    rng = np.random.default_rng(21)
+    n = 5000
+    k1 = (rng.integers(0, 40, n) / 8).astype(np.float32)  # heavy ties on the first key
+    k2 = (rng.integers(0, 1 << 12, n) / 4096).astype(np.float32)
+    k2[::7] = k2[3]  # ties on both keys -> the row id decides
+    for k in (1, 10, 100, 1000):
+        v1, v2, i = oracle.topk_kk(k1, k2, k, l1, l2)
+        ref = lex_ref(k1, k2, k, l1, l2)
+        assert np.array_equal(i, ref)
+        assert v1.tobytes() == k1[ref].tobytes() and v2.tobytes() == k2[ref].tobytes()
+
+
+def test_compound_keys_special_values_brute_force():
+    """Tiny inputs over special floats vs Python's sort of (code1, code2, -idx) tuples
+    built from torch's stable sort ranks (an independent order for NaN / -0)."""
+    sp = np.array([np.nan, -np.inf, -0.0, 0.0, 1.0, np.inf], dtype=np.float32)
+    rng = np.random.default_rng(22)
+    for trial in range(200):
+        n = int(rng.integers(1, 12))
+        k1 = sp[rng.integers(0, sp.shape[0], n)]
+        k2 = sp[rng.integers(0, sp.shape[0], n)]
+        # dense rank of each value under "NaN greatest, -0 == +0" via torch.sort
+        def rank(a):
+            t = torch.from_numpy(a)
+            _, order = torch.sort(t, stable=True)
+            r = np.empty(n, dtype=np.int64)
+            cur = -1
+            prev = None
+            for pos in order.numpy():
+                x = a[pos]
+                same = prev is not None and ((np.isnan(x) and np.isnan(prev)) or x == prev)
+                if not same:
+                    cur += 1
+                r[pos] = cur
+                prev = x
+            return r
+        r1, r2 = rank(k1), rank(k2)
+        for l1 in (True, False):
+            for l2 in (True, False):
+                key = sorted(range(n), key=lambda i: ((-r1[i]) if l1 else r1[i],
+                                                      (-r2[i]) if l2 else r2[i], i))
+                k = int(rng.integers(1, n + 1))
+                _, _, i = oracle.topk_kk(k1, k2, k, l1, l2)
+                assert list(i) == key[:k], (k1, k2, l1, l2)
+
+
+def test_compound_keys_reduce_to_single_key():
+    """Constant second key: the single-key oracle (pinned above) decides."""
+    rng = np.random.default_rng(23)
+    k1 = rng.random(3000, dtype=np.float32)
+    k2 = np.full(3000, 0.25, dtype=np.float32)
+    for l1 in (True, False):
+        _, _, i = oracle.topk_kk(k1, k2, 64, l1, True)
+        _, si = oracle.topk(k1, 64, l1)
+        assert np.array_equal(i, si)
