@@ -152,6 +152,25 @@ topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank
                          uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
                          void* stream);
 
+/* Compound keys -- "two keys + value (KKV)" (§6.6):
+ *   SELECT row WHERE pred(row) ORDER BY keys1 [DESC|ASC], keys2 [DESC|ASC] LIMIT k
+ * Lexicographic: keys1 decides (order1), keys2 breaks its ties (order2), then the lowest
+ * row id; each column uses topk_select's float order (NaN greatest, -0 == +0).  The
+ * value is the tuple id carried through the network and gathered at the end
+ * ("pass around the tuple id and construct the full tuple at the end"):
+ * out_idx, and out_payload = payload[row] if payload is given.  Both key columns stream
+ * through the same single pass (8 bytes per row; 12 with a predicate).
+ *   keys1, keys2  DEVICE float [n], 16-byte aligned; pred / payload as topk_query.
+ *   out_keys1/2   DEVICE float [k] (either may be NULL); rows beyond the matches of a
+ *                 predicate get out_idx = -1 and zero bits.
+ *   ws            topk_workspace_bytes(TOPK_F64, n, k) bytes (12-byte entries).
+ *   1 <= k <= min(n, 1024); n <= 2^32 - 2. */
+topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t* pred,
+                      const uint32_t* payload, uint64_t n, uint32_t k, topk_order_t order1,
+                      topk_order_t order2, float* out_keys1, float* out_keys2,
+                      uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
+                      void* stream);
+
 /* Top-k of keys in HOST memory (pinned memory strongly recommended): the input is
  * streamed to the device in chunks of `chunk_keys` keys through a double-buffered
  * staging area inside `ws`; each chunk's top-k runs as soon as it has landed, so the

@@ -213,7 +213,9 @@ int oracle_certificate(int dtype, const void* keys, uint64_t n, uint64_t base, u
  *   column, e.g. "lang = 'en' OR lang = 'es'").
  * f (reading R18): rank_b == NULL -> f = keys[i] (any dtype); else (f32 only)
  *   f = keys[i] + w * rank_b[i], the product and the sum each rounded to float
- *   ("retweet_count + 0.5 * likes_count"; built with -ffp-contract=off).
+ *   ("retweet_count + 0.5 * likes_count"; built with -ffp-contract=off); a NaN
+ *   result is returned as the canonical quiet NaN 0x7FC00000 (IEEE-754 leaves the
+ *   payload of a computed NaN open; it ranks the same either way).
  * Plain plan: (1) filter + project into a new array with the source row ids, (2)
  * oracle_topk over it with explicit indices.  Rows beyond the number of matches get
  * out_idx = -1 and all-zero key bits.  Returns the number of result rows (<= k), or
@@ -239,6 +241,10 @@ int oracle_query(int dtype, const void* keys, const float* rank_b, float w, int 
             const float prod = w * rank_b[i];
             const float f = a + prod;
             std::memcpy(b, &f, 4);
+            if (std::isnan(f)) {  // R18: a computed NaN is returned as the canonical 0x7FC00000
+                const uint32_t qnan = 0x7FC00000u;
+                std::memcpy(b, &qnan, 4);
+            }
         } else {
             std::memcpy(b, static_cast<const char*>(keys) + kb * i, kb);
         }

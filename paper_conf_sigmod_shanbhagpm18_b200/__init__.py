@@ -18,7 +18,7 @@ import torch
 
 from . import _lib
 
-__all__ = ["topk", "topk_host", "merge", "query", "Workspace", "launch_count", "workspace_bytes"]
+__all__ = ["topk", "topk_host", "merge", "query", "topk_kk", "Workspace", "launch_count", "workspace_bytes"]
 
 _DT = {torch.float32: _lib.F32, torch.uint32: _lib.U32, torch.float64: _lib.F64}
 
@@ -153,6 +153,49 @@ def query(keys: torch.Tensor, k: int, largest: bool = True, rank_b: torch.Tensor
                         _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(keys.device))
     _lib.check(st, "topk_query")
     return (vals, idx) if payload is None else (vals, idx, pay)
+
+
+def _pred_struct(pred, n):
+    if pred is None:
+        return None
+    if pred[1].dtype != torch.uint32 or pred[1].shape[0] != n or not pred[1].is_contiguous():
+        raise ValueError("predicate column: contiguous CUDA uint32 of the same length")
+    if pred[0] == "range":
+        return _lib.Pred(_lib.PRED_RANGE, pred[1].data_ptr(), int(pred[2]), int(pred[3]), 0)
+    if pred[0] == "in":
+        return _lib.Pred(_lib.PRED_IN, pred[1].data_ptr(), 0, 0, int(pred[2]))
+    raise ValueError(f"unknown predicate kind {pred[0]!r}")
+
+
+def topk_kk(k1: torch.Tensor, k2: torch.Tensor, k: int, largest1: bool = True,
+            largest2: bool = True, pred: tuple | None = None,
+            payload: torch.Tensor | None = None, workspace: Workspace | None = None):
+    """Compound-key top-k, ``ORDER BY k1, k2 LIMIT k`` over two CUDA float32 columns
+    (KKV), lexicographic, ties to the lowest row.  Returns
+    ``(v1, v2, indices)`` or ``(v1, v2, indices, payload_out)``."""
+    if not (k1.is_cuda and k2.is_cuda) or k1.dim() != 1 or k1.shape != k2.shape:
+        raise ValueError("topk_kk expects two 1-D CUDA float32 tensors of one length")
+    if k1.dtype != torch.float32 or k2.dtype != torch.float32:
+        raise TypeError("topk_kk: float32 key columns")
+    lib = _lib.load()
+    n = k1.shape[0]
+    pr = _pred_struct(pred, n)
+    dev = k1.device
+    v1 = torch.empty(k, dtype=torch.float32, device=dev)
+    v2 = torch.empty(k, dtype=torch.float32, device=dev)
+    idx = torch.empty(k, dtype=torch.int64, device=dev)
+    pay = torch.empty(k, dtype=torch.uint32, device=dev) if payload is not None else None
+    need = int(lib.topk_workspace_bytes(_lib.F64, n, k))
+    if need == 0:
+        raise _lib.TopkError(f"invalid arguments for topk_kk (n={n}, k={k})")
+    ws = workspace if workspace is not None else _workspace(dev, need)
+    st = lib.topk_kk(_ptr(k1.contiguous()), _ptr(k2.contiguous()),
+                     ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k,
+                     _lib.LARGEST if largest1 else _lib.SMALLEST,
+                     _lib.LARGEST if largest2 else _lib.SMALLEST, _ptr(v1), _ptr(v2), _ptr(pay),
+                     _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(dev))
+    _lib.check(st, "topk_kk")
+    return (v1, v2, idx) if payload is None else (v1, v2, idx, pay)
 
 
 def topk_host(x: torch.Tensor, k: int, largest: bool = True, chunk_keys: int = 1 << 26,

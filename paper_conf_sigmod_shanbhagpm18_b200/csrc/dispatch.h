@@ -31,6 +31,7 @@ TOPK_DECLARE_SELECT_TU(f64)
 TOPK_DECLARE_QUERY_TU(f32)
 TOPK_DECLARE_QUERY_TU(u32)
 TOPK_DECLARE_QUERY_TU(f64)
+TOPK_DECLARE_QUERY_TU(kk)
 #undef TOPK_DECLARE_QUERY_TU
 
 }  // namespace topk

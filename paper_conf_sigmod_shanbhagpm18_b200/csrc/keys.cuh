@@ -227,4 +227,30 @@ struct KeyTraits<double> {
     }
 };
 
+// Compound key (two f32 columns a, b, ORDER BY a, b -- KKV; R19):
+// a tag type for the select kernel's query form kQKey2.  The entry is E64 with the
+// 64-bit code (code(a) << 32) | code2(b): one unsigned compare is the lexicographic
+// order, the row id breaks the remaining ties.  The streamed a column is read as
+// float4 like f32 keys; the kernel computes codes directly (no threshold key).
+struct KK32 {
+    float a;
+};
+template <>
+struct KeyTraits<KK32> {
+    using Key = KK32;
+    using E = E64;
+    using Vec = float4;
+    static constexpr int kVec = 4;
+    template <bool MIN>
+    __device__ __forceinline__ static KK32 decode(uint64_t) {
+        return KK32{0.f};  // unused: the compound fast test compares codes
+    }
+    // (code(a) << 32) | code(b): a in the kernel's order, b in order2 (1 = ascending)
+    template <bool MIN>
+    __device__ __forceinline__ static uint64_t code2(float a, float b, uint32_t b_min) {
+        const uint32_t cb = KeyTraits<float>::code_max(b);
+        return (static_cast<uint64_t>(KeyTraits<float>::code<MIN>(a)) << 32) | (b_min ? ~cb : cb);
+    }
+};
+
 }  // namespace topk

@@ -66,7 +66,9 @@ using CSync = NamedSync<kNC>;
 
 template <class Key>
 struct Cfg {
-    static constexpr int kStages = sizeof(Key) == 8 ? TOPK_STAGES - 1 : TOPK_STAGES;
+    // 12-byte entries (E64: f64 and compound keys) leave room for one stage less
+    static constexpr int kStages =
+        std::is_same<typename KeyTraits<Key>::E, E64>::value ? TOPK_STAGES - 1 : TOPK_STAGES;
     static constexpr int kTileKeys = kTileBytes / static_cast<int>(sizeof(Key));
     static constexpr int kVecPerThread = kTileBytes / 16 / kNC;
     static constexpr int kItems = kTileKeys / kNC;  // keys per consumer thread per tile
@@ -76,18 +78,19 @@ struct Cfg {
 // Query forms (the paper's §5 database integration; R17/R18): the
 // streamed row is more than the key column.  Q bits: kQPred -- a u32 predicate column
 // (WHERE), kQRank -- a second f32 column b with the ranking function f = a + w * b
-// (ORDER BY f).  A ring stage then holds one slab per column, TK rows each.
-constexpr int kQPred = 1, kQRank = 2;
+// (ORDER BY f), kQKey2 -- a second f32 key column b (Key = KK32: ORDER BY a, b).  A ring
+// stage then holds one slab per column, TK rows each.
+constexpr int kQPred = 1, kQRank = 2, kQKey2 = 4;
 template <class Key, int Q>
 struct QCfg {
-    static constexpr int kRowBytes = static_cast<int>(sizeof(Key)) + ((Q & kQRank) ? 4 : 0) +
-                                     ((Q & kQPred) ? 4 : 0);
+    static constexpr int kRowBytes = static_cast<int>(sizeof(Key)) +
+                                     ((Q & (kQRank | kQKey2)) ? 4 : 0) + ((Q & kQPred) ? 4 : 0);
     static constexpr int kItems =
         Q == 0 ? Cfg<Key>::kItems : (kRowBytes <= 8 ? 8 : 4);  // rows per consumer thread
     static constexpr int kTileKeys = Q == 0 ? Cfg<Key>::kTileKeys : kNC * kItems;
     static constexpr int kVecPerThread = kItems / KeyTraits<Key>::kVec;
-    static constexpr int kOffB = kTileKeys * static_cast<int>(sizeof(Key));  // rank column b
-    static constexpr int kOffP = kOffB + ((Q & kQRank) ? kTileKeys * 4 : 0);  // predicate
+    static constexpr int kOffB = kTileKeys * static_cast<int>(sizeof(Key));  // column b
+    static constexpr int kOffP = kOffB + ((Q & (kQRank | kQKey2)) ? kTileKeys * 4 : 0);  // pred
     static_assert(Q == 0 || kTileKeys * kRowBytes <= kTileBytes, "stage size");
     static_assert(kTileKeys % 4 == 0, "TMA sizes are multiples of 16 bytes");
 };
@@ -122,7 +125,9 @@ struct SelectParams {
     uint32_t gmax;     // workspace layout: published-sample columns (>= gridDim.x)
     uint32_t J;        // published samples per CTA: the 2^j-th best of its run, j < J
     // query forms (Q != 0; select_kernel's template argument)
-    const float* rank_b;   // kQRank: column b of f = key + rank_w * b
+    const float* col_b;    // kQRank: column b of f = key + rank_w * b; kQKey2: second key
+    float* out_keys2;      // kQKey2: b of each result row
+    uint32_t order2_min;   // kQKey2: b ascending (1) or descending (0)
     const uint32_t* pred;  // kQPred: predicate column
     float rank_w;
     uint32_t pred_in;      // 1: membership (pred < 64 and bit pred of pred_mask); 0: range
@@ -140,8 +145,11 @@ __device__ __forceinline__ bool pred_ok(const SelectParams& p, uint32_t v) {
 }
 // ORDER BY f (reading R18): f = a + w * b, the product and the sum each rounded to
 // nearest f32 (no fused multiply-add, so the oracle's plain C arithmetic agrees).
+// A NaN result is returned as the canonical quiet NaN 0x7FC00000 (IEEE-754 leaves a
+// computed NaN's payload open; the order code of every NaN is the same).
 __device__ __forceinline__ float rank_f(float a, float w, float b) {
-    return __fadd_rn(a, __fmul_rn(w, b));
+    const float f = __fadd_rn(a, __fmul_rn(w, b));
+    return f != f ? __uint_as_float(0x7FC00000u) : f;
 }
 
 // Workspace: [WsHeader | pub: u64[kPubRows][gmax] | cand: G x k entries]
@@ -800,6 +808,62 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
     const int tid = threadIdx.x;
     const int lane = tid & 31;
 
+    auto pos_of = [&](int q) -> uint32_t {
+        return static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
+    };
+    if constexpr ((Q & kQKey2) != 0) {
+        // compound key: 64-bit codes (code(a) << 32 | code2(b)); fast test on the code
+        uint64_t cc[ITEMS];
+        const float4* sa = reinterpret_cast<const float4*>(slot_data);
+        const float4* sb = reinterpret_cast<const float4*>(slot_data + QC::kOffB);
+#pragma unroll
+        for (int j = 0; j < VPT; ++j) {
+            const float4 a = sa[tid + j * kNC], b = sb[tid + j * kNC];
+#pragma unroll
+            for (int w = 0; w < VEC; ++w)
+                cc[j * VEC + w] = KT::template code2<MIN>(vget(a, w), vget(b, w), p.order2_min);
+        }
+        uint32_t mask = (ITEMS >= 32) ? 0xFFFFFFFFu : ((1u << ITEMS) - 1u);
+        if constexpr ((Q & kQPred) != 0) {
+            const uint4* sp = reinterpret_cast<const uint4*>(slot_data + QC::kOffP);
+            uint32_t pm = 0;
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+                const uint4 u = sp[tid + j * kNC];
+#pragma unroll
+                for (int w = 0; w < VEC; ++w)
+                    pm |= static_cast<uint32_t>(pred_ok(p, vget(u, w))) << (j * VEC + w);
+            }
+            mask &= pm;
+        }
+        if (tlen < static_cast<uint32_t>(TK)) {
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                if (pos_of(q) >= tlen) mask &= ~(1u << q);
+        }
+        if (pr.active) {
+            // superset test on the code (>= always valid; > once every row of the tile
+            // comes after the bound's row), then the exact (code, row) test
+            const uint64_t tc = pr.tau.c;
+            const bool strict = lbase > pr.strict_after;
+            uint32_t keep = 0;
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q) {
+                const bool f = strict ? cc[q] > tc : cc[q] >= tc;
+                keep |= static_cast<uint32_t>(f) << q;
+            }
+            mask &= keep;
+            if (!__any_sync(0xFFFFFFFFu, mask != 0u)) return 0;
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                if (((mask >> q) & 1u) && !better(E::make(cc[q], lbase + pos_of(q)), pr.tau))
+                    mask &= ~(1u << q);
+        }
+        E ents[ITEMS];
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q) ents[q] = E::make(cc[q], lbase + pos_of(q));
+        return append<E, ITEMS>(buf, s_cnt, ents, mask, limit);
+    } else {
     Key x[ITEMS];
     {
         const Vec* sv = reinterpret_cast<const Vec*>(slot_data);
@@ -832,9 +896,6 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
                 pm |= static_cast<uint32_t>(pred_ok(p, vget(u, w))) << (j * VEC + w);
         }
     }
-    auto pos_of = [&](int q) -> uint32_t {
-        return static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
-    };
     if (tlen < static_cast<uint32_t>(TK)) {
 #pragma unroll
         for (int q = 0; q < ITEMS; ++q)
@@ -883,15 +944,28 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
     for (int q = 0; q < ITEMS; ++q)
         if ((keep >> q) & 1u) buf.st(w++, E::make(KT::template code<MIN>(x[q]), lbase + pos_of(q)));
     return old;
+    }
 }
 
 // The key of global row `row` under query form Q (the extras and the finalize gather).
 template <class Key, int Q>
 __device__ __forceinline__ Key query_key(const SelectParams& p, const Key* keys, uint64_t row) {
     if constexpr ((Q & kQRank) != 0)
-        return rank_f(keys[row], p.rank_w, p.rank_b[row]);
+        return rank_f(keys[row], p.rank_w, p.col_b[row]);
     else
         return keys[row];
+}
+// The entry of global row `row` (< 2^32 - 1) under query form Q.
+template <class Key, bool MIN, int Q>
+__device__ __forceinline__ typename KeyTraits<Key>::E query_entry(const SelectParams& p,
+                                                                  const Key* keys, uint64_t row) {
+    using KT = KeyTraits<Key>;
+    if constexpr ((Q & kQKey2) != 0)
+        return KT::E::make(KT::template code2<MIN>(keys[row].a, p.col_b[row], p.order2_min),
+                           static_cast<uint32_t>(row));
+    else
+        return KT::E::make(KT::template code<MIN>(query_key<Key, Q>(p, keys, row)),
+                           static_cast<uint32_t>(row));
 }
 
 template <class Key, bool MIN, bool FILTER, int Q = 0>
@@ -975,10 +1049,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             bool ok = tid < nextra;
             if constexpr ((Q & kQPred) != 0) ok = ok && pred_ok(p, p.pred[ok ? row : 0]);
             const uint32_t bal = __ballot_sync(0xFFFFFFFFu, ok);
-            if (ok)
-                buf.st(__popc(bal & ((1u << tid) - 1u)),
-                       E::make(KT::template code<MIN>(query_key<Key, Q>(p, keys, row)),
-                               static_cast<uint32_t>(row)));
+            if (ok) buf.st(__popc(bal & ((1u << tid) - 1u)), query_entry<Key, MIN, Q>(p, keys, row));
             if (tid == 0) st.cnt = __popc(bal);
         }
     }
@@ -1029,8 +1100,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             uint32_t bytes = static_cast<uint32_t>(len * sizeof(Key));
             unsigned char* dst = ring + static_cast<size_t>(slot) * kTileBytes;
             tma_load_1d(dst, body + lo, bytes, &full[slot], policy);
-            if constexpr ((Q & kQRank) != 0) {  // one slab per column (query forms: head == 0)
-                tma_load_1d(dst + QCfg<Key, Q>::kOffB, p.rank_b + lo,
+            if constexpr ((Q & (kQRank | kQKey2)) != 0) {  // one slab per column (head == 0)
+                tma_load_1d(dst + QCfg<Key, Q>::kOffB, p.col_b + lo,
                             static_cast<uint32_t>(len * 4), &full[slot], policy);
                 bytes += static_cast<uint32_t>(len * 4);
             }
@@ -1255,13 +1326,20 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (e.is_sentinel()) {  // fewer than k rows (only a WHERE can do that, since k <= n)
             if (Q == 0) atomicAdd(&g_stats[7], 1ull);  // plain form: a bug
             if (p.out_idx) p.out_idx[j] = -1;
-            if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = Key(0);
+            if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = Key{0};
+            if constexpr ((Q & kQKey2) != 0)
+                if (p.out_keys2) p.out_keys2[j] = 0.f;
             if (p.out_payload) p.out_payload[j] = 0u;
             continue;
         }
         const uint32_t row = e.lidx();
         if (p.out_idx) p.out_idx[j] = static_cast<int64_t>(p.base + row);
-        if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = query_key<Key, Q>(p, keys, row);
+        if constexpr ((Q & kQKey2) != 0) {
+            if (p.out_keys) static_cast<float*>(p.out_keys)[j] = keys[row].a;
+            if (p.out_keys2) p.out_keys2[j] = p.col_b[row];
+        } else {
+            if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = query_key<Key, Q>(p, keys, row);
+        }
         if (p.out_payload) p.out_payload[j] = p.payload[row];
     }
     if (tid == 0) trace(6);

@@ -50,7 +50,17 @@ cudaError_t TOPK_CAT(launch_select_, TOPK_TU_NAME)(const SelectParams& p, int gr
 cudaError_t TOPK_CAT(launch_query_, TOPK_TU_NAME)(const SelectParams& p, int grid,
                                                   bool min_order, int q, cudaStream_t st) {
     using Key = TOPK_TU_KEY;
-    if constexpr (sizeof(Key) == 4 && static_cast<Key>(-1) < static_cast<Key>(0)) {  // f32
+    if constexpr (std::is_same<Key, KK32>::value) {  // compound keys (+ optional WHERE)
+        switch (q) {
+            case kQKey2:
+                return min_order ? launch_one<Key, true, true, kQKey2>(p, grid, st)
+                                 : launch_one<Key, false, true, kQKey2>(p, grid, st);
+            case kQKey2 | kQPred:
+                return min_order ? launch_one<Key, true, true, kQKey2 | kQPred>(p, grid, st)
+                                 : launch_one<Key, false, true, kQKey2 | kQPred>(p, grid, st);
+        }
+        return cudaErrorInvalidValue;
+    } else if constexpr (std::is_same<Key, float>::value) {
         switch (q) {
             case kQPred:
                 return min_order ? launch_one<Key, true, true, kQPred>(p, grid, st)

@@ -85,10 +85,18 @@ cudaError_t dispatch_query(topk_dtype_t dt, const topk::SelectParams& p, int gri
     return e;
 }
 
+cudaError_t dispatch_query_kk(const topk::SelectParams& p, int grid, bool min_order, int q,
+                              cudaStream_t st) {
+    const cudaError_t e = topk::launch_query_kk(p, grid, min_order, q, st);
+    if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
+    return e;
+}
+
 // Every select translation unit's debug accessor (each holds its own device globals).
 int (*const kSelectDebug[])(int, void*, int) = {topk::debug_select_f32, topk::debug_select_u32,
                                                 topk::debug_select_f64, topk::debug_query_f32,
-                                                topk::debug_query_u32, topk::debug_query_f64};
+                                                topk::debug_query_u32, topk::debug_query_f64,
+                                                topk::debug_query_kk};
 
 template <class Key, bool MIN>
 cudaError_t launch_merge(const topk::MergeParams& p, cudaStream_t st) {
@@ -127,6 +135,10 @@ uint32_t query_tile_keys(topk_dtype_t dt, int q) {
     using topk::QCfg;
     using topk::kQPred;
     using topk::kQRank;
+    using topk::kQKey2;
+    if (q & kQKey2)
+        return (q & kQPred) ? QCfg<topk::KK32, kQKey2 | kQPred>::kTileKeys
+                            : QCfg<topk::KK32, kQKey2>::kTileKeys;
     if (dt == TOPK_F64) return QCfg<double, kQPred>::kTileKeys;
     if (dt == TOPK_U32) return QCfg<uint32_t, kQPred>::kTileKeys;
     switch (q) {
@@ -198,6 +210,8 @@ struct QueryArgs {
     const float* rank_b = nullptr;
     float rank_w = 0.f;
     topk_pred_t pred{};
+    float* out_keys2 = nullptr;  // kQKey2
+    uint32_t order2_min = 0;
 };
 
 static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
@@ -237,7 +251,7 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
     p.body_n = qa.q ? n / 4 * 4 : (n - head) / vec * vec;
     const uint32_t tk = qa.q ? query_tile_keys(dtype, qa.q) : tile_keys_for(dtype);
     if (qa.q) {
-        p.rank_b = qa.rank_b;
+        p.col_b = qa.rank_b;
         p.rank_w = qa.rank_w;
         if (qa.q & topk::kQPred) {
             p.pred = qa.pred.col;
@@ -284,6 +298,11 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
+    if (qa.q & topk::kQKey2) {
+        p.out_keys2 = qa.out_keys2;
+        p.order2_min = qa.order2_min;
+        return dispatch_query_kk(p, grid, mn, qa.q, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+    }
     if (qa.q) return dispatch_query(dtype, p, grid, mn, qa.q, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
     return dispatch_select(dtype, p, grid, mn, filt, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
 }
@@ -351,6 +370,33 @@ topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank
         (payload && misaligned(payload)))
         return TOPK_ERR_INVALID_ARG;
     return select_one(dtype, keys, payload, n, 0, k, order, TOPK_MODE_FILTER, out_keys,
+                      out_payload, out_idx, ws, ws_bytes, stream, qa);
+}
+
+topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t* pred,
+                      const uint32_t* payload, uint64_t n, uint32_t k, topk_order_t order1,
+                      topk_order_t order2, float* out_keys1, float* out_keys2,
+                      uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
+                      void* stream) {
+    if (!keys1 || !keys2 || n == 0 || n > kMaxLaunchN) return TOPK_ERR_INVALID_ARG;
+    if (!valid_order(order1) || !valid_order(order2)) return TOPK_ERR_INVALID_ARG;
+    QueryArgs qa;
+    qa.q = topk::kQKey2;
+    qa.rank_b = keys2;
+    qa.out_keys2 = out_keys2;
+    qa.order2_min = order2 == TOPK_SMALLEST ? 1u : 0u;
+    if (pred) {
+        if ((pred->kind != TOPK_PRED_RANGE && pred->kind != TOPK_PRED_IN) || !pred->col)
+            return TOPK_ERR_INVALID_ARG;
+        qa.q |= topk::kQPred;
+        qa.pred = *pred;
+    }
+    auto misaligned = [](const void* c) { return reinterpret_cast<uintptr_t>(c) % 16 != 0; };
+    if (misaligned(keys1) || misaligned(keys2) || (pred && misaligned(pred->col)) ||
+        (payload && misaligned(payload)))
+        return TOPK_ERR_INVALID_ARG;
+    // 12-byte (64-bit code, row) entries: the f64 workspace layout
+    return select_one(TOPK_F64, keys1, payload, n, 0, k, order1, TOPK_MODE_FILTER, out_keys1,
                       out_payload, out_idx, ws, ws_bytes, stream, qa);
 }
 

@@ -152,3 +152,69 @@ def test_full_size_query1(cuda_device):
     keys = datagen.generate("uniform", n, "u32", seed=319)
     t = u32col(n, 320)
     run(keys, 50, True, pred=("range", t, 0, 1 << 31))
+
+
+# ---- compound keys: ORDER BY k1, k2 LIMIT k (KKV) ----
+
+def run_kk(k1, k2, k, l1=True, l2=True, pred=None, payload=None):
+    dev = "cuda"
+    gpred = None if pred is None else (pred[0], pred[1].to(dev), *pred[2:])
+    out = tk.topk_kk(k1.to(dev), k2.to(dev), k, l1, l2, pred=gpred,
+                     payload=None if payload is None else payload.to(dev))
+    torch.cuda.synchronize()
+    h1, h2 = host(k1), host(k2)
+    if pred is None:
+        o1, o2, oi = oracle.topk_kk(h1, h2, k, l1, l2)
+    else:  # the plain plan: filter, then the compound top-k over the survivors
+        c = host(pred[1])
+        keep = (c >= pred[2]) & (c < pred[3]) if pred[0] == "range" else \
+            (c < 64) & (((np.uint64(pred[2]) >> np.minimum(c, 63).astype(np.uint64)) & np.uint64(1)) == 1)
+        rows = np.nonzero(keep)[0]
+        m = min(k, rows.shape[0])
+        oi = np.full(k, -1, dtype=np.int64)
+        o1 = np.zeros(k, dtype=np.float32)
+        o2 = np.zeros(k, dtype=np.float32)
+        if m:
+            a1, a2, ii = oracle.topk_kk(h1[rows], h2[rows], m, l1, l2)
+            oi[:m], o1[:m], o2[:m] = rows[ii], a1, a2
+    gi = out[2].cpu().numpy()
+    assert np.array_equal(gi, oi), f"indices differ: first at {np.nonzero(gi != oi)[0][:5]}"
+    assert host(out[0]).tobytes() == o1.tobytes() and host(out[1]).tobytes() == o2.tobytes()
+    if payload is not None:
+        ph = host(payload)
+        exp = np.where(oi >= 0, ph[np.maximum(oi, 0)], 0).astype(np.uint32)
+        assert np.array_equal(host(out[3]), exp)
+
+
+@pytest.mark.parametrize("l1", [True, False])
+@pytest.mark.parametrize("l2", [True, False])
+def test_compound_keys(cuda_device, l1, l2):
+    k1 = datagen.generate("fewdistinct", N, "f32", seed=321)  # 16 values: k2 decides
+    k2 = datagen.generate("uniform", N, "f32", seed=322)
+    for k in (1, 8, 64, 256, 1024):
+        run_kk(k1, k2, k, l1, l2)
+
+
+def test_compound_keys_ties_and_specials(cuda_device):
+    k1 = datagen.generate("fewdistinct", N, "f32", seed=323)
+    k2 = datagen.generate("fewdistinct", N, "f32", seed=324)  # full ties: row id decides
+    run_kk(k1, k2, 300, True, False)
+    k1 = datagen.generate("uniform", 200000, "f32", seed=325)
+    k2 = datagen.generate("uniform", 200000, "f32", seed=326)
+    for j, (a, b) in enumerate([(float("nan"), 1.0), (float("nan"), float("nan")), (-0.0, 2.0),
+                                (0.0, 2.0), (float("inf"), -float("inf")), (1.0, float("nan"))]):
+        k1[j * 31337] = a
+        k2[j * 31337] = b
+    for l1 in (True, False):
+        for l2 in (True, False):
+            run_kk(k1, k2, 16, l1, l2)
+
+
+@pytest.mark.parametrize("dist", ["uniform", "increasing", "decreasing"])
+def test_compound_keys_predicate_payload(cuda_device, dist):
+    k1 = datagen.generate(dist, N, "f32", seed=327)
+    k2 = datagen.generate("uniform", N, "f32", seed=328)
+    col = u32col(N, 329, 100)
+    pay = datagen.payload(N, seed=330)
+    run_kk(k1, k2, 64, True, True, pred=("range", col, 10, 60), payload=pay)
+    run_kk(k1, k2, 64, False, True, pred=("in", col, (1 << 7) | (1 << 40)), payload=pay)

@@ -23,6 +23,9 @@ def lib_query(a, k, largest, rank_b=None, w=0.0, keep=None):
     """numpy filter + projection, torch stable sort; indices refer to the input rows."""
     rows = np.arange(a.shape[0], dtype=np.int64)
     f = a if rank_b is None else (a + np.float32(w) * rank_b).astype(np.float32)
+    if rank_b is not None:  # R18: computed NaNs are the canonical quiet NaN
+        f = f.copy()
+        f[np.isnan(f)] = np.uint32(0x7FC00000).view(np.float32)
     if keep is not None:
         rows, f = rows[keep], f[keep]
     m = min(k, rows.shape[0])
