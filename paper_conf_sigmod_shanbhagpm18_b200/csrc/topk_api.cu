@@ -61,42 +61,24 @@ bool valid_order(int o) { return o == TOPK_LARGEST || o == TOPK_SMALLEST; }
 // the sentinel entry).
 constexpr uint64_t kMaxLaunchN = 0xFFFFFFFEull;
 
-cudaError_t dispatch_select(topk_dtype_t dt, const topk::SelectParams& p, int grid,
-                            bool min_order, bool filter, cudaStream_t st) {
-    cudaError_t e;
-    switch (dt) {
-        case TOPK_F32: e = topk::launch_select_f32(p, grid, min_order, filter, st); break;
-        case TOPK_U32: e = topk::launch_select_u32(p, grid, min_order, filter, st); break;
-        default: e = topk::launch_select_f64(p, grid, min_order, filter, st); break;
+// One select kernel instantiation per generated TU (dispatch.h kSelectTable).
+cudaError_t launch_variant(int key, bool min_order, bool filter, int q,
+                           const topk::SelectParams& p, int grid, cudaStream_t st) {
+    for (int i = 0; i < topk::kSelectTableN; ++i) {
+        const topk::SelectEntry& v = topk::kSelectTable[i];
+        if (v.key == key && v.min == (min_order ? 1 : 0) && v.filter == (filter ? 1 : 0) &&
+            v.q == q) {
+            const cudaError_t e = v.launch(p, grid, st);
+            if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
+            return e;
+        }
     }
-    if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
-    return e;
+    return cudaErrorInvalidValue;  // no such instantiation
 }
 
-cudaError_t dispatch_query(topk_dtype_t dt, const topk::SelectParams& p, int grid,
-                           bool min_order, int q, cudaStream_t st) {
-    cudaError_t e;
-    switch (dt) {
-        case TOPK_F32: e = topk::launch_query_f32(p, grid, min_order, q, st); break;
-        case TOPK_U32: e = topk::launch_query_u32(p, grid, min_order, q, st); break;
-        default: e = topk::launch_query_f64(p, grid, min_order, q, st); break;
-    }
-    if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
-    return e;
+int key_kind(topk_dtype_t dt) {
+    return dt == TOPK_F64 ? topk::kKeyF64 : dt == TOPK_U32 ? topk::kKeyU32 : topk::kKeyF32;
 }
-
-cudaError_t dispatch_query_kk(const topk::SelectParams& p, int grid, bool min_order, int q,
-                              cudaStream_t st) {
-    const cudaError_t e = topk::launch_query_kk(p, grid, min_order, q, st);
-    if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
-    return e;
-}
-
-// Every select translation unit's debug accessor (each holds its own device globals).
-int (*const kSelectDebug[])(int, void*, int) = {topk::debug_select_f32, topk::debug_select_u32,
-                                                topk::debug_select_f64, topk::debug_query_f32,
-                                                topk::debug_query_u32, topk::debug_query_f64,
-                                                topk::debug_query_kk};
 
 template <class Key, bool MIN>
 cudaError_t launch_merge(const topk::MergeParams& p, cudaStream_t st) {
@@ -301,10 +283,11 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
     if (qa.q & topk::kQKey2) {
         p.out_keys2 = qa.out_keys2;
         p.order2_min = qa.order2_min;
-        return dispatch_query_kk(p, grid, mn, qa.q, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+        return launch_variant(topk::kKeyKK, mn, true, qa.q, p, grid, st) == cudaSuccess
+                   ? TOPK_OK : TOPK_ERR_CUDA;
     }
-    if (qa.q) return dispatch_query(dtype, p, grid, mn, qa.q, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
-    return dispatch_select(dtype, p, grid, mn, filt, st) == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+    return launch_variant(key_kind(dtype), mn, qa.q ? true : filt, qa.q, p, grid, st) == cudaSuccess
+               ? TOPK_OK : TOPK_ERR_CUDA;
 }
 
 
@@ -459,7 +442,8 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
  * select_kernel (flushes, survivors flushed, flush cycles, deferrals, tiles). */
 int topk_debug_stats(uint64_t* host8, int reset) {
     for (int i = 0; i < 8; ++i) host8[i] = 0;
-    for (auto f : kSelectDebug) {
+    for (int i = 0; i < topk::kSelectTableN; ++i) {
+        const auto f = topk::kSelectTable[i].debug;
         if (f(topk::kDbgStatsAdd, host8, 0) != 0) return -1;
         if (reset && f(topk::kDbgStatsReset, nullptr, 0) != 0) return -1;
     }
@@ -536,8 +520,8 @@ int topk_debug_cnet(int e64, const void* d_codes, int n, int Lp, void* d_out) {
 
 /* Debug switches of the select kernel (select.cuh c_dbg), set in every select TU. */
 int topk_debug_flags(int flags) {
-    for (auto f : kSelectDebug)
-        if (f(topk::kDbgFlags, nullptr, flags) != 0) return -1;
+    for (int i = 0; i < topk::kSelectTableN; ++i)
+        if (topk::kSelectTable[i].debug(topk::kDbgFlags, nullptr, flags) != 0) return -1;
     return 0;
 }
 
@@ -549,15 +533,15 @@ int topk_debug_trace(int enable, uint64_t* host) {
     if (host) {
         static uint64_t tmp[kRows * kLen];
         std::memset(host, 0, sizeof(tmp));
-        for (auto f : kSelectDebug) {
-            if (f(topk::kDbgTraceRead, tmp, 0) != 0) return -1;
+        for (int i = 0; i < topk::kSelectTableN; ++i) {
+            if (topk::kSelectTable[i].debug(topk::kDbgTraceRead, tmp, 0) != 0) return -1;
             for (size_t r = 0; r < kRows; ++r)
                 if (tmp[r * kLen] > host[r * kLen])
                     std::memcpy(host + r * kLen, tmp + r * kLen, kLen * sizeof(uint64_t));
         }
     }
-    for (auto f : kSelectDebug)
-        if (f(topk::kDbgTraceSet, nullptr, enable) != 0) return -1;
+    for (int i = 0; i < topk::kSelectTableN; ++i)
+        if (topk::kSelectTable[i].debug(topk::kDbgTraceSet, nullptr, enable) != 0) return -1;
     return 0;
 }
 
