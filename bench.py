@@ -307,7 +307,16 @@ def run_ours(args):
         cfgs.append({"config": "f1 query2: ORDER BY a + 0.5 * b DESC LIMIT 50 (f32 cols)",
                      "us": round(t * 1e3, 1), "rows_per_s": n4 / (t / 1e3),
                      "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
-        del a, b
+        # f3: compound keys, KKV (Fig 14's 2^28 tuples): ORDER BY k1, k2 with the
+        # 4-byte value gathered through the tuple id; 8 bytes streamed per row
+        k1 = datagen.generate("uniform", n4, "f32", seed=datagen.config_seed(7), device=dev)
+        k2 = datagen.generate("uniform", n4, "f32", seed=datagen.config_seed(7, 1), device=dev)
+        pv = datagen.payload(n4, seed=datagen.config_seed(7), device=dev)
+        t = timed(lambda: tk.topk_kk(k1, k2, 64, True, True, payload=pv))
+        cfgs.append({"config": "f3 KKV: 2^28 rows, ORDER BY k1 DESC, k2 DESC LIMIT 64, u32 value",
+                     "us": round(t * 1e3, 1), "rows_per_s": n4 / (t / 1e3),
+                     "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
+        del k1, k2, pv, a, b
         for kk in (32, 256):
             t = timed(lambda: tk.topk(x, kk, True, mode="pure"), 2)
             cfgs.append({"config": f"pure mode (paper's data-independent network on every key), "

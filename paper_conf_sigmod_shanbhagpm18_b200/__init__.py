@@ -18,7 +18,7 @@ import torch
 
 from . import _lib
 
-__all__ = ["topk", "topk_host", "merge", "query", "topk_kk", "Workspace", "launch_count", "workspace_bytes"]
+__all__ = ["topk", "topk_host", "merge", "query", "topk_kk", "topk_radix", "Workspace", "launch_count", "workspace_bytes"]
 
 _DT = {torch.float32: _lib.F32, torch.uint32: _lib.U32, torch.float64: _lib.F64}
 
@@ -196,6 +196,31 @@ def topk_kk(k1: torch.Tensor, k2: torch.Tensor, k: int, largest1: bool = True,
                      _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(dev))
     _lib.check(st, "topk_kk")
     return (v1, v2, idx) if payload is None else (v1, v2, idx, pay)
+
+
+def topk_radix(x: torch.Tensor, k: int, largest: bool = True, out=None):
+    """Radix-select top-k (the paper's selection-based method): the same
+    result as :func:`topk`, by MSD passes over 8-bit digits of the order code."""
+    if not x.is_cuda or x.dim() != 1:
+        raise ValueError("topk_radix expects a 1-D CUDA tensor (no CPU path)")
+    lib = _lib.load()
+    dt = _dtype_code(x)
+    n = x.shape[0]
+    x = x.contiguous()
+    need = int(lib.topk_radix_workspace_bytes(dt, n, k))
+    if need == 0:
+        raise _lib.TopkError(f"invalid arguments for topk_radix (n={n}, k={k})")
+    key = ("radix", x.device.index, torch.cuda.current_stream(x.device).cuda_stream)
+    ws = _ws_cache.get(key)
+    if ws is None or ws.nbytes < need:
+        ws = Workspace(need, x.device)
+        _ws_cache[key] = ws
+    vals, idx = out if out is not None else (torch.empty(k, dtype=x.dtype, device=x.device),
+                                             torch.empty(k, dtype=torch.int64, device=x.device))
+    st = lib.topk_radix(dt, _ptr(x), n, k, _lib.LARGEST if largest else _lib.SMALLEST,
+                        _ptr(vals), _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(x.device))
+    _lib.check(st, "topk_radix")
+    return vals, idx
 
 
 def topk_host(x: torch.Tensor, k: int, largest: bool = True, chunk_keys: int = 1 << 26,

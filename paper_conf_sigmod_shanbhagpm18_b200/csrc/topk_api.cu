@@ -12,6 +12,7 @@
 #include "probe.cuh"
 #include "netbench.cuh"
 #include "dispatch.h"
+#include "radix.cuh"
 #include "select.cuh"
 #include "topk.h"
 
@@ -381,6 +382,69 @@ topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t*
     // 12-byte (64-bit code, row) entries: the f64 workspace layout
     return select_one(TOPK_F64, keys1, payload, n, 0, k, order1, TOPK_MODE_FILTER, out_keys1,
                       out_payload, out_idx, ws, ws_bytes, stream, qa);
+}
+
+// ---- radix-select top-k (radix.cuh; the paper's selection-based method) ----
+struct RadixPlan {
+    uint32_t G, cap;
+    uint64_t slice;
+};
+static RadixPlan radix_plan(uint64_t n, int sms) {
+    RadixPlan r;
+    const uint64_t g = 4ull * static_cast<uint64_t>(sms);  // 4 CTAs of 256 threads per SM
+    uint64_t slice = (n + g - 1) / g;
+    slice = (slice + topk::kRadixTile - 1) / topk::kRadixTile * topk::kRadixTile;
+    r.slice = slice;
+    r.G = static_cast<uint32_t>((n + slice - 1) / slice);
+    uint64_t cap = n / 16;
+    if (cap < 65536) cap = 65536;
+    if (cap > n) cap = n;
+    r.cap = static_cast<uint32_t>(cap);
+    return r;
+}
+
+size_t topk_radix_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k) {
+    if (!valid_dtype(dtype) || n == 0 || k == 0 || k > TOPK_MAX_K || k > n || n > kMaxLaunchN)
+        return 0;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return 0;
+    const RadixPlan r = radix_plan(n, sms);
+    return topk::radix_workspace_bytes(key_kind(dtype), r.G, k, r.cap);
+}
+
+topk_status_t topk_radix(topk_dtype_t dtype, const void* keys, uint64_t n, uint32_t k,
+                         topk_order_t order, void* out_keys, int64_t* out_idx, void* ws,
+                         size_t ws_bytes, void* stream) {
+    if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
+    if (!keys || n == 0 || k == 0 || k > TOPK_MAX_K || k > n || n > kMaxLaunchN)
+        return TOPK_ERR_INVALID_ARG;
+    if (reinterpret_cast<uintptr_t>(keys) % key_size(dtype)) return TOPK_ERR_INVALID_ARG;
+    int sms = 0, major = 0;
+    if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    if (major != 10) return TOPK_ERR_UNSUPPORTED;
+    const RadixPlan r = radix_plan(n, sms);
+    if (!ws || (reinterpret_cast<uintptr_t>(ws) % 256) ||
+        ws_bytes < topk::radix_workspace_bytes(key_kind(dtype), r.G, k, r.cap))
+        return TOPK_ERR_WORKSPACE;
+    topk::RadixParams p;
+    std::memset(&p, 0, sizeof(p));
+    p.keys = keys;
+    p.n = n;
+    p.base = 0;
+    p.k = k;
+    p.K = next_pow2_u32(k);
+    p.G = r.G;
+    p.slice = r.slice;
+    p.cap = r.cap;
+    p.ws = static_cast<unsigned char*>(ws);
+    p.out_keys = out_keys;
+    p.out_idx = out_idx;
+    int launches = 0;
+    const cudaError_t e = topk::launch_radix(key_kind(dtype), order == TOPK_SMALLEST, p,
+                                             static_cast<cudaStream_t>(stream), &launches);
+    if (e != cudaSuccess) return TOPK_ERR_CUDA;
+    g_launches.fetch_add(static_cast<uint64_t>(launches), std::memory_order_relaxed);
+    return TOPK_OK;
 }
 
 topk_status_t topk_f32(const float* keys, uint64_t n, uint32_t k, topk_order_t order,
