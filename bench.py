@@ -251,6 +251,23 @@ def run_ours(args):
             t = time_steps(f, 10, stream, torch) / 10
             sweep.append({"k": kk, "us": round(t * 1e3, 1), "keys_per_s": n / (t / 1e3)})
         extra["k_sweep_uniform"] = sweep
+        # f2: the paper's selection-based method (radix select) on the same
+        # input, next to the §7 cost model's predictions with B200 parameters
+        from paper_conf_sigmod_shanbhagpm18_b200 import costmodel as cm
+        hw = cm.b200(peaks()[0])
+        rv = []
+        for kk in (32, 256, 1024):
+            f = lambda: tk.topk_radix(x, kk, True)
+            for _ in range(3):
+                f()
+            t = time_steps(f, 10, stream, torch) / 10
+            tb = next(s_["us"] for s_ in sweep if s_["k"] == kk)
+            rv.append({"k": kk, "radix_us": round(t * 1e3, 1), "bitonic_us": tb,
+                       "model_radix_us": round(cm.radix_time(n, KEY_BYTES, hw) * 1e6, 1),
+                       "model_bitonic_paper_us": round(cm.bitonic_time(n, KEY_BYTES, kk, hw) * 1e6, 1),
+                       "model_choice": cm.choose(n, KEY_BYTES, kk, hw),
+                       "measured_choice": "bitonic" if tb <= t * 1e3 else "radix"})
+        extra["radix_vs_bitonic"] = rv
         adv = []
         for d in ("increasing", "decreasing", "fewdistinct", "bucketkiller"):
             xa = datagen.generate(d, n, "f32", seed=datagen.config_seed(3), device=dev)

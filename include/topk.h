@@ -176,8 +176,8 @@ topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t*
  * larger K") and of its cost model (§7.1).  Same result as topk_select
  * (R1-R5: identical values, rows and order).  MSD passes over 8-bit digits of
  * the order code (4 for 32-bit keys, 8 for f64): histogram -> prefix sum -> the bucket
- * holding the k-th best; the digit-1 bucket is written once (if it fits the workspace)
- * together with the entries of higher digits, later digits read only the bucket; ties
+ * holding the k-th best; the bucket is written once, at the first digit where it fits
+ * the workspace, with every entry above it; later digits read only the bucket; ties
  * at the k-th code resolve to the lowest rows (a further input pass when the ties do
  * not fit).  At least two reads of the input (histogram + bucket pass), against one
  * for topk_select -- the reason the bench's dispatch keeps bitonic top-k on B200.
@@ -185,7 +185,7 @@ topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t*
  *   ws        topk_radix_workspace_bytes(dtype, n, k) bytes (O(n / 16 * entry): the
  *             bucket; cf. "selection-based methods require an additional buffer",
  *             P:209), 256-byte aligned, zero-filled before first use; left zeroed.
- *   Enqueues 10 (32-bit keys) or 18 (f64) kernels on `stream`, no host sync. */
+ *   Enqueues 15 (32-bit keys) or 27 (f64) kernels on `stream`, no host sync. */
 size_t topk_radix_workspace_bytes(topk_dtype_t dtype, uint64_t n, uint32_t k);
 topk_status_t topk_radix(topk_dtype_t dtype, const void* keys, uint64_t n, uint32_t k,
                          topk_order_t order, void* out_keys, int64_t* out_idx, void* ws,

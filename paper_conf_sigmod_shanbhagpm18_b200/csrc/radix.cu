@@ -26,6 +26,7 @@ cudaError_t radix_seq(const RadixParams& p, cudaStream_t st) {
     for (int d = 1; d < static_cast<int>(sizeof(C)); ++d) {  // the remaining digits
         radix_hist<Key, MIN, false><<<G, kRadixNT, 0, st>>>(p);
         radix_choose<C, false><<<1, kRadixBins, 0, st>>>(p);
+        radix_scatter<Key, MIN><<<G, kRadixNT, 0, st>>>(p);
     }
     radix_collect<C><<<G, kRadixNT, 0, st>>>(p);
     radix_emit<Key, MIN><<<G, kRadixNT, 0, st>>>(p);
@@ -38,7 +39,7 @@ cudaError_t radix_seq(const RadixParams& p, cudaStream_t st) {
 cudaError_t launch_radix(int key, bool min_order, const RadixParams& p, cudaStream_t st,
                          int* launches) {
     const int nd = key == kKeyF64 ? 8 : 4;
-    *launches = 3 + 2 * (nd - 1) + 3;
+    *launches = 3 * nd + 3;
     switch (key) {
         case kKeyF32: return min_order ? radix_seq<float, true>(p, st) : radix_seq<float, false>(p, st);
         case kKeyU32:

@@ -8,13 +8,14 @@
 //     by the known prefix, or the bucket) -> prefix sum from the top -> the digit d_j
 //     of the bucket holding the k-th best code ("uses the histogram to find the bucket
 //     B containing the k-th-largest entry");
-//   after digit 1, "writes out only the entries of B" -- here the bucket
-//     is written once (scatter) if it fits the workspace; else "the clustering step is
-//     skipped and we simply re-use the input in the next pass";
+//   "writes out only the entries of B" -- here the bucket is written
+//     once (scatter), after the first digit whose bucket fits the workspace; before
+//     that "the clustering step is skipped and we simply re-use the input in the next
+//     pass" -- U(0,1) floats put half the keys in one first-digit bucket;
 //   "when scanning the array the second time to write out the tuples that fall into
 //     the bucket, we can also write out the elements in the higher buckets to a
-//     separate result array" -- the scatter pass appends digit > d_1 entries
-//     to the result candidates.
+//     separate result array" -- the scatter pass appends every entry above
+//     the bucket to the result candidates.
 // After the last digit the k-th best code X is known exactly.  The result is every
 // entry with code > X plus the lowest-index entries with code == X (the tie rule of
 // DESIGN.md R1 -- the paper pads "with X", which fixes values but not rows):
@@ -51,11 +52,13 @@ struct RadixState {
     C prefix;            // known top digits of X (bits above `shift`)
     uint32_t shift;      // bit position of the next digit
     uint32_t k_rem;      // rank of X inside the current candidates (1-based)
-    uint32_t bucket_ok;  // 1: the digit-1 bucket was written (later passes read it)
+    uint32_t bucket_ok;  // 1: a bucket was written (later passes read it)
     uint32_t nbucket;    // entries written to the bucket
     uint32_t ngt;        // result candidates with code > X (exactly k - m at the end)
     uint32_t neq;        // ties (code == X) collected from the bucket
     uint32_t need_emit;  // 1: the final input pass collects gt / ties
+    uint32_t scatter;    // 1: the bucket of the digit just chosen is written next
+    uint32_t bshift;     // bit position of the digit just chosen
     uint32_t pad;
 };
 
@@ -204,6 +207,16 @@ __device__ __forceinline__ void warp_append(RadixEntry<C>* list, uint32_t* cnt, 
     }
 }
 
+// Shared-memory histogram increment, aggregated over the lanes holding the same digit
+// (one atomic per distinct digit per warp: U(0,1) floats put half the keys on one
+// first digit, and same-address atomics serialise).
+__device__ __forceinline__ void hist_add(uint32_t* h, uint32_t digit, bool valid) {
+    const uint32_t act = __ballot_sync(0xFFFFFFFFu, valid);
+    if (!valid) return;
+    const uint32_t peers = __match_any_sync(act, digit);
+    if ((threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&h[digit], __popc(peers));
+}
+
 // Digit pass: per-CTA histogram of digit `shift` over the candidates -- the input
 // filtered by the known prefix (pass 1, or when the bucket was not written), else the
 // bucket.  Counts only; the choice is made by radix_choose.
@@ -219,9 +232,12 @@ __global__ void __launch_bounds__(kRadixNT) radix_hist(const RadixParams p) {
     __syncthreads();
     if (from_bucket) {
         const uint32_t nb = w.st->nbucket;
-        for (uint32_t i = blockIdx.x * kRadixNT + threadIdx.x; i < nb; i += gridDim.x * kRadixNT) {
-            const C c = w.bucket[i].code;
-            if (has_prefix(c, prefix, shift)) atomicAdd(&h[digit_of(c, shift)], 1u);
+        const uint32_t stride = gridDim.x * kRadixNT;
+        const uint32_t n_iter = (nb + stride - 1) / stride;
+        for (uint32_t it = 0; it < n_iter; ++it) {
+            const uint32_t i = it * stride + blockIdx.x * kRadixNT + threadIdx.x;
+            const C c = i < nb ? w.bucket[i].code : C(0);
+            hist_add(h, digit_of(c, shift), i < nb && has_prefix(c, prefix, shift));
         }
     } else {
         const Key* keys = static_cast<const Key*>(p.keys);
@@ -232,8 +248,7 @@ __global__ void __launch_bounds__(kRadixNT) radix_hist(const RadixParams p) {
             const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
 #pragma unroll
             for (int q = 0; q < kRadixPerThread; ++q)
-                if (r0 + q < hi && has_prefix(c[q], prefix, shift))
-                    atomicAdd(&h[digit_of(c[q], shift)], 1u);
+                hist_add(h, digit_of(c[q], shift), r0 + q < hi && has_prefix(c[q], prefix, shift));
         }
     }
     __syncthreads();
@@ -255,14 +270,18 @@ __global__ void __launch_bounds__(kRadixBins) radix_choose(const RadixParams p) 
     for (uint32_t c = 0; c < p.G; ++c) s += w.hist[static_cast<size_t>(c) * kRadixBins + d];
     tot[d] = s;
     __syncthreads();
-    if (FIRST && d == 0) {
-        st->prefix = 0;
-        st->shift = sizeof(C) * 8 - 8;
-        st->k_rem = p.k;
-        st->nbucket = 0;
-        st->ngt = 0;
-        st->neq = 0;
-        st->need_emit = 0;
+    if (d == 0) {
+        if (FIRST) {
+            st->prefix = 0;
+            st->shift = sizeof(C) * 8 - 8;
+            st->k_rem = p.k;
+            st->nbucket = 0;
+            st->ngt = 0;
+            st->neq = 0;
+            st->need_emit = 0;
+            st->bucket_ok = 0;
+        }
+        st->scatter = 0;
     }
     __syncthreads();
     // above[d] = sum of tot over digits > d: inclusive scan from the top
@@ -277,21 +296,28 @@ __global__ void __launch_bounds__(kRadixBins) radix_choose(const RadixParams p) 
         const uint32_t shift = st->shift;
         st->prefix = st->prefix | (static_cast<C>(dig) << shift);
         st->k_rem = kr - above;
-        if (FIRST) st->bucket_ok = v <= p.cap ? 1u : 0u;
+        // write the bucket once, as soon as it fits the workspace ("if after the prefix
+        // sum we see no data reduction, the clustering step is skipped")
+        if (!st->bucket_ok && v <= p.cap) {
+            st->scatter = 1;
+            st->bucket_ok = 1;
+        }
+        st->bshift = shift;
         st->shift = shift >= 8 ? shift - 8 : 0;
         if (shift == 0) st->shift = 0xFFFFFFFFu;  // done: prefix == X
     }
 }
 
-// After digit 1: write the bucket (entries with digit d_1) and append the entries of
-// higher digits to the result.  Skipped (exits) if the bucket does not fit.
+// After the digit whose bucket first fits the workspace: write the bucket (entries
+// whose code carries the prefix chosen so far) and append every entry above it to the
+// result.  Exits at once at the other digits.
 template <class Key, bool MIN>
 __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
     using C = typename CodeOf<typename KeyTraits<Key>::E>::C;
     const RadixWs<C> w = radix_ws<C>(p.ws, p.G, p.k);
-    if (!w.st->bucket_ok) return;
-    constexpr uint32_t kTop = sizeof(C) * 8 - 8;
-    const uint32_t d1 = static_cast<uint32_t>(w.st->prefix >> kTop);
+    if (!w.st->scatter) return;
+    const uint32_t kTop = w.st->bshift;
+    const C d1 = w.st->prefix >> kTop;
     const Key* keys = static_cast<const Key*>(p.keys);
     const uint64_t lo = blockIdx.x * p.slice, hi = min(p.n, lo + p.slice);
     for (uint64_t t0 = lo; t0 < hi; t0 += kRadixTile) {
@@ -301,7 +327,7 @@ __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
 #pragma unroll
         for (int q = 0; q < kRadixPerThread; ++q) {
             const bool ok = r0 + q < hi;
-            const uint32_t dg = static_cast<uint32_t>(c[q] >> kTop);
+            const C dg = c[q] >> kTop;  // code above the bucket's bits
             const RadixEntry<C> e{c[q], static_cast<uint32_t>(r0 + q)};
             warp_append(w.gt, &w.st->ngt, p.k, ok && dg > d1, e, nullptr);
             warp_append(w.bucket, &w.st->nbucket, p.cap, ok && dg == d1, e, nullptr);
@@ -437,6 +463,7 @@ __global__ void __launch_bounds__(kMergeNT, 1) radix_final(const RadixParams p) 
         st->nbucket = 0;
         st->need_emit = 0;
         st->bucket_ok = 0;
+        st->scatter = 0;
     }
 }
 
