@@ -207,53 +207,59 @@ __device__ __forceinline__ void warp_append(RadixEntry<C>* list, uint32_t* cnt, 
     }
 }
 
-// Shared-memory histogram increment, aggregated over the lanes holding the same digit
-// (one atomic per distinct digit per warp: U(0,1) floats put half the keys on one
-// first digit, and same-address atomics serialise).
-__device__ __forceinline__ void hist_add(uint32_t* h, uint32_t digit, bool valid) {
-    const uint32_t act = __ballot_sync(0xFFFFFFFFu, valid);
-    if (!valid) return;
-    const uint32_t peers = __match_any_sync(act, digit);
-    if ((threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&h[digit], __popc(peers));
-}
-
 // Digit pass: per-CTA histogram of digit `shift` over the candidates -- the input
-// filtered by the known prefix (pass 1, or when the bucket was not written), else the
-// bucket.  Counts only; the choice is made by radix_choose.
+// filtered by the known prefix (pass 1, or while no bucket was written), else the
+// bucket.  Counts only; the choice is made by radix_choose.  Counters are private per
+// lane (u16 [warp][bin][lane]: bank = lane, no atomics, no conflicts) -- U(0,1) floats
+// put half the keys on one first digit, where shared atomics would serialise.  A lane
+// counts at most slice / kHistNT < 2^16 keys (radix_plan).
+constexpr int kHistNT = 128;
+constexpr size_t kHistSmem = size_t(kHistNT / 32) * kRadixBins * 32 * sizeof(uint16_t);  // 64 KB
 template <class Key, bool MIN, bool FIRST>
-__global__ void __launch_bounds__(kRadixNT) radix_hist(const RadixParams p) {
+__global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
     using C = typename CodeOf<typename KeyTraits<Key>::E>::C;
-    __shared__ uint32_t h[kRadixBins];
+    extern __shared__ __align__(16) uint16_t hl[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const RadixWs<C> w = radix_ws<C>(p.ws, p.G, p.k);
-    for (int i = threadIdx.x; i < kRadixBins; i += kRadixNT) h[i] = 0;
+    {
+        uint4* z = reinterpret_cast<uint4*>(hl);
+        for (int i = threadIdx.x; i < static_cast<int>(kHistSmem / 16); i += kHistNT)
+            z[i] = make_uint4(0u, 0u, 0u, 0u);
+    }
+    uint16_t* mine = hl + static_cast<size_t>(warp) * kRadixBins * 32 + lane;
     const C prefix = FIRST ? C(0) : w.st->prefix;
     const uint32_t shift = FIRST ? sizeof(C) * 8 - 8 : w.st->shift;
     const bool from_bucket = !FIRST && w.st->bucket_ok;
     __syncthreads();
     if (from_bucket) {
         const uint32_t nb = w.st->nbucket;
-        const uint32_t stride = gridDim.x * kRadixNT;
-        const uint32_t n_iter = (nb + stride - 1) / stride;
-        for (uint32_t it = 0; it < n_iter; ++it) {
-            const uint32_t i = it * stride + blockIdx.x * kRadixNT + threadIdx.x;
-            const C c = i < nb ? w.bucket[i].code : C(0);
-            hist_add(h, digit_of(c, shift), i < nb && has_prefix(c, prefix, shift));
+        for (uint32_t i = blockIdx.x * kHistNT + threadIdx.x; i < nb; i += gridDim.x * kHistNT) {
+            const C c = w.bucket[i].code;
+            if (has_prefix(c, prefix, shift)) mine[digit_of(c, shift) * 32] += 1;
         }
     } else {
         const Key* keys = static_cast<const Key*>(p.keys);
         const uint64_t lo = blockIdx.x * p.slice, hi = min(p.n, lo + p.slice);
-        for (uint64_t t0 = lo; t0 < hi; t0 += kRadixTile) {
+        constexpr int kT = kHistNT * kRadixPerThread;
+        for (uint64_t t0 = lo; t0 < hi; t0 += kT) {
             C c[kRadixPerThread];
-            load_codes<Key, MIN>(keys, hi, t0 + threadIdx.x * kRadixPerThread, c);
             const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
+            load_codes<Key, MIN>(keys, hi, r0, c);
 #pragma unroll
             for (int q = 0; q < kRadixPerThread; ++q)
-                hist_add(h, digit_of(c[q], shift), r0 + q < hi && has_prefix(c[q], prefix, shift));
+                if (r0 + q < hi && has_prefix(c[q], prefix, shift)) mine[digit_of(c[q], shift) * 32] += 1;
         }
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < kRadixBins; i += kRadixNT)
-        w.hist[static_cast<size_t>(blockIdx.x) * kRadixBins + i] = h[i];
+    for (int b = threadIdx.x; b < kRadixBins; b += kHistNT) {
+        uint32_t s = 0;
+        for (int wv = 0; wv < kHistNT / 32; ++wv) {
+            const uint16_t* row = hl + (static_cast<size_t>(wv) * kRadixBins + b) * 32;
+#pragma unroll 8
+            for (int l = 0; l < 32; ++l) s += row[(l + b) & 31];  // rotate: spread banks
+        }
+        w.hist[static_cast<size_t>(blockIdx.x) * kRadixBins + b] = s;
+    }
 }
 
 // Prefix sum from the top digit down: the bucket d holding the k_rem-th best code

@@ -87,6 +87,31 @@ def main(rnd):
         with open(os.path.join(PROF, f"ncu_select_k{k}_{rnd}.md"), "w") as f:
             f.write("\n".join(lines) + "\n")
         traffic[f"select_k{k}"] = rd + wr
+    # other captures: prof_<tag>_<round>.ncu-rep + gpurun_out/prof_meta.json
+    # {tag: {"desc", "cmd", "alg_bytes"}}
+    meta_p = os.path.join(OUT, "prof_meta.json")
+    meta = json.load(open(meta_p)) if os.path.exists(meta_p) else {}
+    for tag, m in meta.items():
+        rep = os.path.join(OUT, f"prof_{tag}_{rnd}.ncu-rep")
+        if not os.path.exists(rep):
+            continue
+        d = raw(rep)
+        lines = [f"# ncu --set full: {m['desc']} ({rnd})", "", f"Command: `{m['cmd']}` (cold-cache, "
+                 "replayed ~40x: compare shares, not absolute times).", "",
+                 "| metric | unit | value |", "|---|---|---|"]
+        for key in KEYS:
+            if key in d:
+                lines.append(f"| {key} | {d[key][1]} | {d[key][0]} |")
+        st = stalls(rep)
+        lines += ["", "Top warp-stall reasons (pc samples):", "",
+                  "| reason | samples |", "|---|---|"] + [f"| {a} | {b} |" for a, b in st.items()]
+        rd = to_bytes(*d["dram__bytes_read.sum"])
+        wr = to_bytes(*d["dram__bytes_write.sum"])
+        lines += ["", f"DRAM traffic per launch: {rd + wr:.4g} B (algorithmic: "
+                      f"{m['alg_bytes']:.4g} B)."]
+        with open(os.path.join(PROF, f"ncu_{tag}_{rnd}.md"), "w") as f:
+            f.write("\n".join(lines) + "\n")
+        traffic[tag] = rd + wr
     with open(traffic_path, "w") as f:
         json.dump(traffic, f, indent=1)
     lp = os.path.join(OUT, f"launches_{rnd}.csv")
