@@ -324,21 +324,64 @@ __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
     if (!w.st->scatter) return;
     const uint32_t kTop = w.st->bshift;
     const C d1 = w.st->prefix >> kTop;
+    // bucket entries are staged in shared memory and written with one global
+    // reservation per flush (a per-warp atomic on one counter serialises in L2)
+    constexpr int kStage = 2048;
+    __shared__ RadixEntry<C> stage[kStage];
+    __shared__ uint32_t s_w[kRadixNT / 32];
+    __shared__ uint32_t s_base;
+    uint32_t staged = 0;
+    auto flush = [&]() {
+        if (threadIdx.x == 0) s_base = atomicAdd(&w.st->nbucket, staged);
+        __syncthreads();
+        const uint32_t base = s_base;
+        for (uint32_t i = threadIdx.x; i < staged; i += kRadixNT)
+            if (base + i < p.cap) w.bucket[base + i] = stage[i];
+        __syncthreads();
+        staged = 0;
+    };
     const Key* keys = static_cast<const Key*>(p.keys);
     const uint64_t lo = blockIdx.x * p.slice, hi = min(p.n, lo + p.slice);
     for (uint64_t t0 = lo; t0 < hi; t0 += kRadixTile) {
         C c[kRadixPerThread];
         const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
         load_codes<Key, MIN>(keys, hi, r0, c);
+        uint32_t nb = 0;
 #pragma unroll
         for (int q = 0; q < kRadixPerThread; ++q) {
             const bool ok = r0 + q < hi;
             const C dg = c[q] >> kTop;  // code above the bucket's bits
-            const RadixEntry<C> e{c[q], static_cast<uint32_t>(r0 + q)};
-            warp_append(w.gt, &w.st->ngt, p.k, ok && dg > d1, e, nullptr);
-            warp_append(w.bucket, &w.st->nbucket, p.cap, ok && dg == d1, e, nullptr);
+            nb += (ok && dg == d1) ? 1u : 0u;
+            // entries above the bucket: fewer than k in all (rare: warp-aggregated)
+            warp_append(w.gt, &w.st->ngt, p.k, ok && dg > d1,
+                        RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)}, nullptr);
         }
+        uint32_t tile_nb;
+        const uint32_t off = block_excl_scan(nb, s_w, &tile_nb);
+        if (tile_nb == 0) continue;
+        if (staged + tile_nb > kStage) flush();
+        if (tile_nb > kStage) {  // a tile mostly in the bucket (e.g. sorted input): direct
+            if (threadIdx.x == 0) s_base = atomicAdd(&w.st->nbucket, tile_nb);
+            __syncthreads();
+            uint32_t at = s_base + off;
+#pragma unroll
+            for (int q = 0; q < kRadixPerThread; ++q)
+                if (r0 + q < hi && (c[q] >> kTop) == d1) {
+                    if (at < p.cap) w.bucket[at] = RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)};
+                    ++at;
+                }
+            __syncthreads();
+            continue;
+        }
+        uint32_t pos = staged + off;
+#pragma unroll
+        for (int q = 0; q < kRadixPerThread; ++q)
+            if (r0 + q < hi && (c[q] >> kTop) == d1)
+                stage[pos++] = RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)};
+        staged += tile_nb;
+        __syncthreads();
     }
+    if (staged) flush();
 }
 
 // After the last digit (prefix == X): from the bucket, entries with code > X join the
