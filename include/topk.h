@@ -16,7 +16,8 @@
  *     index).  code(): NaN (any sign/payload) ranks above +inf and all NaNs tie; -0 and
  *     +0 tie; TOPK_SMALLEST reverses the key order but keeps "lowest index first".
  *   - out[0..k) is best first; out_keys[j] is bit-identical to keys[out_idx[j] - base].
- *   - any 1 <= k <= min(n, 1024) (k need not be a power of two).
+ *   - any 1 <= k <= min(n, 2048) (k need not be a power of two; the paper evaluates
+ *     1..1024, and its shared-memory form holds k <= 2048).
  *
  * Conventions for every call below:
  *   - Pointers named keys/payload/out_* and ws are DEVICE pointers (cudaMalloc or
@@ -48,11 +49,11 @@ extern "C" {
 #endif
 
 #define TOPK_ABI_VERSION 1
-#define TOPK_MAX_K 1024
+#define TOPK_MAX_K 2048
 
 typedef enum {
     TOPK_OK = 0,
-    TOPK_ERR_INVALID_ARG = 1, /* NULL input, k == 0, k > n, k > 1024, bad enum, alias  */
+    TOPK_ERR_INVALID_ARG = 1, /* NULL input, k == 0, k > n, k > 2048, bad enum, alias  */
     TOPK_ERR_UNSUPPORTED = 2, /* device is not sm_100 (B200)                          */
     TOPK_ERR_WORKSPACE = 3,   /* ws NULL, too small or misaligned                      */
     TOPK_ERR_CUDA = 4,        /* a CUDA runtime call or kernel launch failed           */
@@ -136,7 +137,7 @@ topk_status_t topk_f64_kv(const double* keys, const uint32_t* payload, uint64_t 
  *   row id, the order of topk_select), out_idx[j] its row id; when fewer than k rows
  *   match, rows j >= matches get out_idx = -1, out_keys = 0 bits, out_payload = 0.
  *   Layout: every column (keys, rank_b, pred->col, payload) 16-byte aligned, same n;
- *   1 <= k <= min(n, 1024); n <= 2^32 - 2.  Workspace: topk_workspace_bytes(dtype, n, k).
+ *   1 <= k <= min(n, 2048); n <= 2^32 - 2.  Workspace: topk_workspace_bytes(dtype, n, k).
  *   Errors: TOPK_ERR_INVALID_ARG for a misaligned column, a bad predicate kind, rank_b
  *   with a non-F32 dtype, or neither pred nor rank_b (use topk_select). */
 typedef enum { TOPK_PRED_RANGE = 1, TOPK_PRED_IN = 2 } topk_pred_kind_t;
@@ -164,7 +165,7 @@ topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank
  *   out_keys1/2   DEVICE float [k] (either may be NULL); rows beyond the matches of a
  *                 predicate get out_idx = -1 and zero bits.
  *   ws            topk_workspace_bytes(TOPK_F64, n, k) bytes (12-byte entries).
- *   1 <= k <= min(n, 1024); n <= 2^32 - 2. */
+ *   1 <= k <= min(n, 2048); n <= 2^32 - 2. */
 topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t* pred,
                       const uint32_t* payload, uint64_t n, uint32_t k, topk_order_t order1,
                       topk_order_t order2, float* out_keys1, float* out_keys2,
@@ -211,7 +212,7 @@ topk_status_t topk_select_host(topk_dtype_t dtype, const void* h_keys, uint64_t 
  * the exact top-k of `runs` candidate lists of `run_len` entries each, laid out
  * back to back: cand_keys[runs*run_len] (key type), cand_idx[runs*run_len] int64
  * global row ids (the tie-break), cand_payload optional.  Entries may be in any order;
- * duplicated (key, idx) entries are not allowed.  1 <= k <= min(runs*run_len, 1024),
+ * duplicated (key, idx) entries are not allowed.  1 <= k <= min(runs*run_len, 2048),
  * runs*run_len <= 65536.  Single-CTA merge + rebuild network; ws as topk_merge_ws_bytes. */
 size_t topk_merge_workspace_bytes(topk_dtype_t dtype, uint32_t runs, uint32_t run_len,
                                   uint32_t k);

@@ -241,13 +241,18 @@ __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
         const Key* keys = static_cast<const Key*>(p.keys);
         const uint64_t lo = blockIdx.x * p.slice, hi = min(p.n, lo + p.slice);
         constexpr int kT = kHistNT * kRadixPerThread;
-        for (uint64_t t0 = lo; t0 < hi; t0 += kT) {
-            C c[kRadixPerThread];
-            const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
+        // two tiles per iteration, both loaded before either is counted (bytes in flight)
+        for (uint64_t t0 = lo; t0 < hi; t0 += 2 * kT) {
+            C c[kRadixPerThread], c2[kRadixPerThread];
+            const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread, r1 = r0 + kT;
             load_codes<Key, MIN>(keys, hi, r0, c);
+            load_codes<Key, MIN>(keys, hi, r1, c2);
 #pragma unroll
             for (int q = 0; q < kRadixPerThread; ++q)
                 if (r0 + q < hi && has_prefix(c[q], prefix, shift)) mine[digit_of(c[q], shift) * 32] += 1;
+#pragma unroll
+            for (int q = 0; q < kRadixPerThread; ++q)
+                if (r1 + q < hi && has_prefix(c2[q], prefix, shift)) mine[digit_of(c2[q], shift) * 32] += 1;
         }
     }
     __syncthreads();

@@ -59,7 +59,7 @@ constexpr int kNT = kNC + 32;                               // + one producer wa
 constexpr int kTileBytes = kNC * 16 * TOPK_VEC_PER_THREAD;  // 30 KB per TMA stage
 constexpr int kStagesMax = TOPK_STAGES;
 constexpr int kCap = 4096;            // survivor buffer entries (incl. the running run)
-constexpr int kPubRows = 11;          // published 2^j-th best for j <= log2(1024)
+constexpr int kPubRows = 11;          // published 2^j-th best for j <= 10 (k up to 2048)
 constexpr int kGMax = 160;            // CTAs (>= SM count)
 constexpr int kScratch = kPubRows * kGMax;  // shared: staged samples (u64)
 using CSync = NamedSync<kNC>;

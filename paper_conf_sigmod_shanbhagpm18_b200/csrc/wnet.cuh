@@ -1,4 +1,5 @@
-// wnet.cuh -- register/warp-shuffle form of the paper's operators for K <= 256.
+// wnet.cuh -- register/warp-shuffle form of the paper's operators (K <= 2048; bits >= 9
+// of the element index through shared memory).
 //
 // The paper fuses its operators into kernels whose steps run in shared memory
 // ("Operating in Shared Memory") and then combines several steps per thread
@@ -159,10 +160,10 @@ __device__ __forceinline__ void wsmem_step(const SBuf<E>& b, int P, int bb, int 
     Sync::sync();
 }
 
-// Bitonic top-K (K = 2^L <= 1024) of b[0..P), P a power of two, 2K <= P <= 4096, by
+// Bitonic top-K (K = 2^L <= 2048) of b[0..P), P a power of two, 2K <= P <= 4096, by
 // the NW warps of the calling group (warp index w, lane), all of which call this.
 // Result: b[0..K) best first.  Sync is the group's barrier.  Steps on element bits
-// 0-8 run in registers / shuffles; the rare bit-9 steps (K = 1024) in shared memory.
+// 0-8 run in registers / shuffles; the rare steps on bits 9-10 (K >= 1024) in shared memory.
 template <class E, int NW, class Sync>
 __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
     constexpr int RA = 16;  // phase A: 512 entries per warp chunk
@@ -215,9 +216,12 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
     }
     Sync::sync();
     if (threadIdx.x == 0) g_wnet_phase_a_end = clock64();
-    if (L == 10) {  // last local-sort stage (len 512): bit 9 in smem, bits 8..0 in registers
-        wsmem_step<E, NW * 32, Sync>(b, P, 9, 10);
-        wchunk_steps<E, NW>(b, P, 8, 10, w, lane);
+    // local-sort stages beyond 512-runs (len 512, 1024): bits >= 9 in smem, 8..0 in registers
+#pragma unroll 1
+    for (int d = 10; d <= L; ++d) {
+#pragma unroll 1
+        for (int bb = d - 1; bb >= 9; --bb) wsmem_step<E, NW * 32, Sync>(b, P, bb, d);
+        wchunk_steps<E, NW>(b, P, 8, d, w, lane);
         Sync::sync();
     }
     if (L >= 9) {
@@ -245,7 +249,8 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
             }
             Sync::sync();
             P = half;
-            if (L == 10) wsmem_step<E, NW * 32, Sync>(b, P, 9, 10);
+#pragma unroll 1
+            for (int bb = L - 1; bb >= 9; --bb) wsmem_step<E, NW * 32, Sync>(b, P, bb, L);
             wchunk_steps<E, NW>(b, P, 8, L, w, lane);
             Sync::sync();
         }

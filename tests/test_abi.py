@@ -52,7 +52,7 @@ def test_host_only_calls(lib):
                            None, 0, None) == 1
     assert lib.topk_select(0, ctypes.c_void_p(16), None, 10, 0, 11, 0, 0, None, None, None,
                            None, 0, None) == 1
-    assert lib.topk_select(0, ctypes.c_void_p(16), None, 2000, 0, 1025, 0, 0, None, None, None,
+    assert lib.topk_select(0, ctypes.c_void_p(16), None, 5000, 0, 2049, 0, 0, None, None, None,
                            None, 0, None) == 1
     assert lib.topk_select(0, ctypes.c_void_p(18), None, 10, 0, 1, 0, 0, None, None, None,
                            None, 0, None) == 1  # misaligned f32 pointer

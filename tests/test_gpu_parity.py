@@ -51,7 +51,7 @@ def test_config1_uniform_2p20_k32(cuda_device):
 
 
 @pytest.mark.parametrize("k", [1, 2, 3, 7, 8, 31, 32, 33, 64, 100, 128, 255, 256, 257, 512,
-                               777, 1000, 1024])
+                               777, 1000, 1024, 1025, 1500, 2047, 2048])
 def test_every_k_ragged(cuda_device, k):
     n = (1 << 16) + 4096 * 3 + 13  # several tiles + ragged tail
     x = datagen.generate("uniform", n, "f32", seed=101)
@@ -65,7 +65,7 @@ def test_every_k_ragged(cuda_device, k):
 def test_distributions(cuda_device, dist, largest):
     n = (1 << 20) + 13
     x = datagen.generate(dist, n, "f32", seed=202)
-    for k in (1, 64, 256, 1024):
+    for k in (1, 64, 256, 1024, 2048):
         check(x, k, largest)
     check(x, 256, largest, mode="pure")
 

@@ -61,7 +61,7 @@ def test_range_predicate_selectivities(cuda_device, dt, largest):
             run(keys, k, largest, pred=("range", col, lo, hi))
 
 
-@pytest.mark.parametrize("k", [1, 7, 32, 64, 100, 256, 512, 1024])
+@pytest.mark.parametrize("k", [1, 7, 32, 64, 100, 256, 512, 1024, 2048])
 def test_every_k_in_predicate(cuda_device, k):
     keys = datagen.generate("uniform", N, "f32", seed=303)
     lang = u32col(N, 304, 70)  # dictionary codes; >= 64 never match
@@ -191,7 +191,7 @@ def run_kk(k1, k2, k, l1=True, l2=True, pred=None, payload=None):
 def test_compound_keys(cuda_device, l1, l2):
     k1 = datagen.generate("fewdistinct", N, "f32", seed=321)  # 16 values: k2 decides
     k2 = datagen.generate("uniform", N, "f32", seed=322)
-    for k in (1, 8, 64, 256, 1024):
+    for k in (1, 8, 64, 256, 1024, 2048):
         run_kk(k1, k2, k, l1, l2)
 
 

@@ -34,7 +34,7 @@ def check(x_cpu, k, largest=True, offset=0):
 N = (1 << 20) + 4096 * 5 + 11
 
 
-@pytest.mark.parametrize("k", [1, 2, 31, 32, 100, 256, 257, 1000, 1024])
+@pytest.mark.parametrize("k", [1, 2, 31, 32, 100, 256, 257, 1000, 1024, 1500, 2048])
 def test_every_k(cuda_device, k):
     x = datagen.generate("uniform", N, "f32", seed=401)
     check(x, k, True)
