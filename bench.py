@@ -244,7 +244,7 @@ def run_ours(args):
     extra = {}
     if rank == 0 and not args.no_sweep:
         sweep = []
-        for kk in (1, 8, 32, 64, 128, 256, 512, 1024):
+        for kk in (1, 8, 32, 64, 128, 256, 512, 1024, 2048):
             f = lambda: tk.topk(x, kk, True)
             for _ in range(3):
                 f()

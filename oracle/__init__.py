@@ -56,6 +56,8 @@ def _load():
         lib.oracle_query.restype = i32
         lib.oracle_topk_kk.argtypes = [vp, vp, u64, u32, i32, i32, vp, vp, vp]
         lib.oracle_topk_kk.restype = i32
+        lib.oracle_topk_kkk.argtypes = [vp, vp, vp, u64, u32, i32, i32, i32, vp, vp, vp, vp]
+        lib.oracle_topk_kkk.restype = i32
         lib.oracle_threads.argtypes = []
         lib.oracle_threads.restype = i32
         _lib = lib
@@ -143,6 +145,21 @@ def topk_kk(k1: np.ndarray, k2: np.ndarray, k: int, largest1: bool = True,
     if r < 0:
         raise ValueError("oracle_topk_kk: invalid arguments")
     return o1, o2, oi
+
+
+def topk_kkk(k1, k2, k3, k: int, largest=(True, True, True)):
+    """Three compound keys (KKKV): ORDER BY k1, k2, k3 LIMIT k.  Returns
+    ``(v1, v2, v3, indices)``."""
+    cols = [np.ascontiguousarray(c, dtype=np.float32) for c in (k1, k2, k3)]
+    assert cols[0].shape == cols[1].shape == cols[2].shape
+    outs = [np.empty(k, dtype=np.float32) for _ in range(3)]
+    oi = np.empty(k, dtype=np.int64)
+    r = _load().oracle_topk_kkk(*[_ptr(c) for c in cols], cols[0].shape[0], k,
+                                *[0 if l else 1 for l in largest], *[_ptr(o) for o in outs],
+                                _ptr(oi))
+    if r < 0:
+        raise ValueError("oracle_topk_kkk: invalid arguments")
+    return outs[0], outs[1], outs[2], oi
 
 
 def certificate(keys: np.ndarray, k: int, out_keys: np.ndarray, out_idx: np.ndarray,

@@ -297,6 +297,42 @@ int oracle_topk_kk(const float* k1, const float* k2, uint64_t n, uint32_t k, int
     return 0;
 }
 
+/* Three compound keys -- "three keys + value (KKKV)" (§6.6; R19):
+ * ORDER BY k1, k2, k3 LIMIT k, lexicographic on the three columns' codes, then the
+ * lowest row id (the plain rule, written out like oracle_topk_kk). */
+int oracle_topk_kkk(const float* k1, const float* k2, const float* k3, uint64_t n, uint32_t k,
+                    int order1, int order2, int order3, float* out_k1, float* out_k2,
+                    float* out_k3, int64_t* out_idx) {
+    if (!k1 || !k2 || !k3 || n == 0 || k == 0 || k > n) return -1;
+    for (int o : {order1, order2, order3})
+        if (o != 0 && o != 1) return -1;
+    struct Row {
+        uint64_t c1, c2, c3, idx;
+    };
+    std::vector<Row> v(n);
+    for (uint64_t i = 0; i < n; ++i) {
+        v[i].c1 = code_of(DT_F32, k1, i, order1);
+        v[i].c2 = code_of(DT_F32, k2, i, order2);
+        v[i].c3 = code_of(DT_F32, k3, i, order3);
+        v[i].idx = i;
+    }
+    auto lex_better = [](const Row& a, const Row& b) {
+        if (a.c1 != b.c1) return a.c1 > b.c1;
+        if (a.c2 != b.c2) return a.c2 > b.c2;
+        if (a.c3 != b.c3) return a.c3 > b.c3;
+        return a.idx < b.idx;
+    };
+    std::partial_sort(v.begin(), v.begin() + k, v.end(), lex_better);
+    for (uint32_t j = 0; j < k; ++j) {
+        const uint64_t r = v[j].idx;
+        if (out_idx) out_idx[j] = static_cast<int64_t>(r);
+        if (out_k1) std::memcpy(out_k1 + j, k1 + r, 4);
+        if (out_k2) std::memcpy(out_k2 + j, k2 + r, 4);
+        if (out_k3) std::memcpy(out_k3 + j, k3 + r, 4);
+    }
+    return 0;
+}
+
 /* Order code of each key (exposed so tests can pin the code map itself against
  * IEEE-754 facts and against library sorts). */
 void oracle_codes(int dtype, const void* keys, uint64_t n, int order, uint64_t* out) {

@@ -205,3 +205,28 @@ def test_compound_keys_reduce_to_single_key():
         _, _, i = oracle.topk_kk(k1, k2, 64, l1, True)
         _, si = oracle.topk(k1, 64, l1)
         assert np.array_equal(i, si)
+
+
+@pytest.mark.parametrize("orders", [(True, True, True), (False, True, False), (True, False, True)])
+def test_three_keys_vs_lexsort(orders):
+    """KKKV: numpy.lexsort on three NaN-free tie-heavy columns."""
+    rng = np.random.default_rng(24)
+    n = 4000
+    cols = [(rng.integers(0, m, n) / m).astype(np.float32) for m in (6, 5, 50)]
+    sk = [-c.astype(np.float64) if l else c.astype(np.float64) for c, l in zip(cols, orders)]
+    for k in (1, 17, 300, 2048):
+        ref = np.lexsort((np.arange(n), sk[2], sk[1], sk[0]))[:k]
+        v1, v2, v3, i = oracle.topk_kkk(*cols, k, orders)
+        assert np.array_equal(i, ref)
+        assert v3.tobytes() == cols[2][ref].tobytes()
+
+
+def test_three_keys_reduce_to_two():
+    """A constant third key: the (pinned) two-key oracle decides."""
+    rng = np.random.default_rng(25)
+    a = (rng.integers(0, 9, 3000) / 9).astype(np.float32)
+    b = rng.random(3000, dtype=np.float32)
+    c = np.zeros(3000, dtype=np.float32)
+    _, _, _, i = oracle.topk_kkk(a, b, c, 100, (True, False, True))
+    _, _, i2 = oracle.topk_kk(a, b, 100, True, False)
+    assert np.array_equal(i, i2)
