@@ -172,6 +172,16 @@ topk_status_t topk_kk(const float* keys1, const float* keys2, const topk_pred_t*
                       uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
                       void* stream);
 
+/* Three compound keys -- "three keys + value (KKKV)" (§6.6): as topk_kk with
+ * a third float column keys3 (order3) breaking the remaining ties; 12 bytes streamed per
+ * row (16 with a predicate).  ws: topk_workspace_bytes(TOPK_F64, n, k) bytes. */
+topk_status_t topk_kkk(const float* keys1, const float* keys2, const float* keys3,
+                       const topk_pred_t* pred, const uint32_t* payload, uint64_t n, uint32_t k,
+                       topk_order_t order1, topk_order_t order2, topk_order_t order3,
+                       float* out_keys1, float* out_keys2, float* out_keys3,
+                       uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream);
+
 /* Radix-select top-k: the paper's selection-based method (§2.3 "Radix Select", P:93;
  * §4.2), the comparison point of its evaluation ("Radix Select for
  * larger K") and of its cost model (§7.1).  Same result as topk_select

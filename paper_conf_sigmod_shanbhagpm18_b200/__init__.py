@@ -18,7 +18,7 @@ import torch
 
 from . import _lib
 
-__all__ = ["topk", "topk_host", "merge", "query", "topk_kk", "topk_radix", "Workspace", "launch_count", "workspace_bytes"]
+__all__ = ["topk", "topk_host", "merge", "query", "topk_kk", "topk_kkk", "topk_radix", "Workspace", "launch_count", "workspace_bytes"]
 
 _DT = {torch.float32: _lib.F32, torch.uint32: _lib.U32, torch.float64: _lib.F64}
 
@@ -196,6 +196,35 @@ def topk_kk(k1: torch.Tensor, k2: torch.Tensor, k: int, largest1: bool = True,
                      _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(dev))
     _lib.check(st, "topk_kk")
     return (v1, v2, idx) if payload is None else (v1, v2, idx, pay)
+
+
+def topk_kkk(k1: torch.Tensor, k2: torch.Tensor, k3: torch.Tensor, k: int,
+             largest=(True, True, True), pred: tuple | None = None,
+             payload: torch.Tensor | None = None, workspace: Workspace | None = None):
+    """Three compound keys, ``ORDER BY k1, k2, k3 LIMIT k`` (KKKV).  Returns
+    ``(v1, v2, v3, indices)`` or ``(v1, v2, v3, indices, payload_out)``."""
+    cols = (k1, k2, k3)
+    if any(not c.is_cuda or c.dim() != 1 or c.shape != k1.shape or c.dtype != torch.float32
+           for c in cols):
+        raise ValueError("topk_kkk expects three 1-D CUDA float32 tensors of one length")
+    lib = _lib.load()
+    n = k1.shape[0]
+    pr = _pred_struct(pred, n)
+    dev = k1.device
+    outs = [torch.empty(k, dtype=torch.float32, device=dev) for _ in range(3)]
+    idx = torch.empty(k, dtype=torch.int64, device=dev)
+    pay = torch.empty(k, dtype=torch.uint32, device=dev) if payload is not None else None
+    need = int(lib.topk_workspace_bytes(_lib.F64, n, k))
+    if need == 0:
+        raise _lib.TopkError(f"invalid arguments for topk_kkk (n={n}, k={k})")
+    ws = workspace if workspace is not None else _workspace(dev, need)
+    o = [_lib.LARGEST if l else _lib.SMALLEST for l in largest]
+    st = lib.topk_kkk(*[_ptr(c.contiguous()) for c in cols],
+                      ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k, *o,
+                      *[_ptr(t) for t in outs], _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
+                      _stream_ptr(dev))
+    _lib.check(st, "topk_kkk")
+    return (*outs, idx) if payload is None else (*outs, idx, pay)
 
 
 def topk_radix(x: torch.Tensor, k: int, largest: bool = True, out=None):

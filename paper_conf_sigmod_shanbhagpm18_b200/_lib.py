@@ -25,7 +25,7 @@ SYMBOLS = (
     "topk_launch_count", "topk_status_string", "topk_abi_version", "topk_probe_read",
     "topk_host_workspace_bytes", "topk_select_host", "topk_nccl_unique_id", "topk_nccl_comm_init",
     "topk_nccl_comm_destroy", "topk_sharded_workspace_bytes", "topk_select_sharded",
-    "topk_f32_sharded", "topk_query", "topk_kk", "topk_radix_workspace_bytes", "topk_radix",
+    "topk_f32_sharded", "topk_query", "topk_kk", "topk_kkk", "topk_radix_workspace_bytes", "topk_radix",
 )
 PRED_RANGE, PRED_IN = 1, 2
 
@@ -98,6 +98,9 @@ def load(build_if_missing: bool = True):
     lib.topk_kk.argtypes = [vp, vp, ctypes.POINTER(Pred), vp, u64, u32, i32, i32, vp, vp, vp, vp,
                             vp, sz, vp]
     lib.topk_kk.restype = i32
+    lib.topk_kkk.argtypes = [vp, vp, vp, ctypes.POINTER(Pred), vp, u64, u32, i32, i32, i32, vp, vp,
+                             vp, vp, vp, vp, sz, vp]
+    lib.topk_kkk.restype = i32
     lib.topk_radix_workspace_bytes.argtypes = [i32, u64, u32]
     lib.topk_radix_workspace_bytes.restype = sz
     lib.topk_radix.argtypes = [i32, vp, u64, u32, i32, vp, vp, vp, sz, vp]

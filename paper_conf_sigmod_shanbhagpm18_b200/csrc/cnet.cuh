@@ -39,9 +39,14 @@ template <>
 struct CodeOf<E64> {
     using C = uint64_t;
 };
+template <>
+struct CodeOf<E96> {  // the first 64 bits (keys 1 and 2): a code bound on them is valid
+    using C = uint64_t;
+};
 
 __device__ __forceinline__ uint32_t ecode(E32 e) { return static_cast<uint32_t>(e.v >> 32); }
 __device__ __forceinline__ uint64_t ecode(E64 e) { return e.c; }
+__device__ __forceinline__ uint64_t ecode(E96 e) { return e.c; }
 
 __device__ __forceinline__ uint32_t cmax(uint32_t a, uint32_t b) { return max(a, b); }
 __device__ __forceinline__ uint32_t cmin(uint32_t a, uint32_t b) { return min(a, b); }

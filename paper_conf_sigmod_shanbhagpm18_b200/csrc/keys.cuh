@@ -43,6 +43,27 @@ __device__ __forceinline__ bool better(E64 a, E64 b) {
     return a.c > b.c || (a.c == b.c && a.ni > b.ni);
 }
 
+// E96 -- three compound f32 keys (KKKV, R19): {c = code(k1) << 32 | code(k2),
+// c3 = code(k3), ~lidx}, compared lexicographically; sentinel = {0, 0, 0}.
+struct E96 {
+    uint64_t c;
+    uint32_t c3;
+    uint32_t ni;
+    __device__ __forceinline__ static E96 make(uint64_t code, uint32_t code3, uint32_t lidx) {
+        return E96{code, code3, ~lidx};
+    }
+    __device__ __forceinline__ static E96 sentinel() { return E96{0ull, 0u, 0u}; }
+    __device__ __forceinline__ bool is_sentinel() const { return c == 0ull && c3 == 0u && ni == 0u; }
+    __device__ __forceinline__ uint32_t lidx() const { return ~ni; }
+    __device__ __forceinline__ uint64_t code() const { return c; }
+};
+__device__ __forceinline__ bool better(E96 a, E96 b) {
+    // (c3, ni) as one 64-bit word: c3 decides, then the lower row (larger ~lidx)
+    const uint64_t la = (static_cast<uint64_t>(a.c3) << 32) | a.ni;
+    const uint64_t lb = (static_cast<uint64_t>(b.c3) << 32) | b.ni;
+    return a.c > b.c || (a.c == b.c && la > lb);
+}
+
 // Branch-free select (selp): the compiler otherwise turns data-dependent swaps into
 // divergent branches, serialising the warp.
 __device__ __forceinline__ uint64_t sel64(bool p, uint64_t a, uint64_t b) {
@@ -62,6 +83,9 @@ __device__ __forceinline__ uint32_t sel32(bool p, uint32_t a, uint32_t b) {
 __device__ __forceinline__ E32 esel(bool p, E32 a, E32 b) { return E32{sel64(p, a.v, b.v)}; }
 __device__ __forceinline__ E64 esel(bool p, E64 a, E64 b) {
     return E64{sel64(p, a.c, b.c), sel32(p, a.ni, b.ni)};
+}
+__device__ __forceinline__ E96 esel(bool p, E96 a, E96 b) {
+    return E96{sel64(p, a.c, b.c), sel32(p, a.c3, b.c3), sel32(p, a.ni, b.ni)};
 }
 
 // Shared-memory arrays of entries (structure of arrays for E64: 12 B per entry).
@@ -122,6 +146,43 @@ struct SBuf<E64> {
     __device__ __forceinline__ void st2(int i, E64 a, E64 b) const {
         const int j = swz(i);
         *reinterpret_cast<ulonglong2*>(c + j) = make_ulonglong2(a.c, b.c);
+        *reinterpret_cast<uint2*>(ni + j) = make_uint2(a.ni, b.ni);
+    }
+};
+
+template <>
+struct SBuf<E96> {
+    uint64_t* c;
+    uint32_t* c3;
+    uint32_t* ni;
+    static constexpr int kBytes = 16;
+    __device__ __forceinline__ void init(unsigned char* base, int cap) {
+        c = reinterpret_cast<uint64_t*>(base);
+        c3 = reinterpret_cast<uint32_t*>(base + 8 * static_cast<size_t>(cap));
+        ni = reinterpret_cast<uint32_t*>(base + 12 * static_cast<size_t>(cap));
+    }
+    __device__ __forceinline__ E96 ld(int i) const {
+        const int j = swz(i);
+        return E96{c[j], c3[j], ni[j]};
+    }
+    __device__ __forceinline__ void st(int i, E96 e) const {
+        const int j = swz(i);
+        c[j] = e.c;
+        c3[j] = e.c3;
+        ni[j] = e.ni;
+    }
+    __device__ __forceinline__ void ld2(int i, E96& a, E96& b) const {
+        const int j = swz(i);
+        const ulonglong2 q = *reinterpret_cast<const ulonglong2*>(c + j);
+        const uint2 t = *reinterpret_cast<const uint2*>(c3 + j);
+        const uint2 n = *reinterpret_cast<const uint2*>(ni + j);
+        a = E96{q.x, t.x, n.x};
+        b = E96{q.y, t.y, n.y};
+    }
+    __device__ __forceinline__ void st2(int i, E96 a, E96 b) const {
+        const int j = swz(i);
+        *reinterpret_cast<ulonglong2*>(c + j) = make_ulonglong2(a.c, b.c);
+        *reinterpret_cast<uint2*>(c3 + j) = make_uint2(a.c3, b.c3);
         *reinterpret_cast<uint2*>(ni + j) = make_uint2(a.ni, b.ni);
     }
 };
@@ -250,6 +311,31 @@ struct KeyTraits<KK32> {
     __device__ __forceinline__ static uint64_t code2(float a, float b, uint32_t b_min) {
         const uint32_t cb = KeyTraits<float>::code_max(b);
         return (static_cast<uint64_t>(KeyTraits<float>::code<MIN>(a)) << 32) | (b_min ? ~cb : cb);
+    }
+};
+
+// Three compound keys (a, b, c; KKKV): tag type of the select kernel's query form
+// kQKey2 | kQKey3, entry E96.
+struct KKK32 {
+    float a;
+};
+template <>
+struct KeyTraits<KKK32> {
+    using Key = KKK32;
+    using E = E96;
+    using Vec = float4;
+    static constexpr int kVec = 4;
+    template <bool MIN>
+    __device__ __forceinline__ static KKK32 decode(uint64_t) {
+        return KKK32{0.f};  // unused: the compound fast test compares codes
+    }
+    template <bool MIN>
+    __device__ __forceinline__ static uint64_t code2(float a, float b, uint32_t b_min) {
+        return KeyTraits<KK32>::code2<MIN>(a, b, b_min);
+    }
+    __device__ __forceinline__ static uint32_t code3(float c, uint32_t c_min) {
+        const uint32_t cc = KeyTraits<float>::code_max(c);
+        return c_min ? ~cc : cc;
     }
 };
 

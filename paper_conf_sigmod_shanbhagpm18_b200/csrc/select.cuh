@@ -67,8 +67,11 @@ using CSync = NamedSync<kNC>;
 template <class Key>
 struct Cfg {
     // 12-byte entries (E64: f64 and compound keys) leave room for one stage less
+    // (16-byte entries, E96: three compound keys, two less)
     static constexpr int kStages =
-        std::is_same<typename KeyTraits<Key>::E, E64>::value ? TOPK_STAGES - 1 : TOPK_STAGES;
+        std::is_same<typename KeyTraits<Key>::E, E96>::value   ? TOPK_STAGES - 2
+        : std::is_same<typename KeyTraits<Key>::E, E64>::value ? TOPK_STAGES - 1
+                                                               : TOPK_STAGES;
     static constexpr int kTileKeys = kTileBytes / static_cast<int>(sizeof(Key));
     static constexpr int kVecPerThread = kTileBytes / 16 / kNC;
     static constexpr int kItems = kTileKeys / kNC;  // keys per consumer thread per tile
@@ -80,17 +83,20 @@ struct Cfg {
 // (WHERE), kQRank -- a second f32 column b with the ranking function f = a + w * b
 // (ORDER BY f), kQKey2 -- a second f32 key column b (Key = KK32: ORDER BY a, b).  A ring
 // stage then holds one slab per column, TK rows each.
-constexpr int kQPred = 1, kQRank = 2, kQKey2 = 4;
+// kQKey3 -- a third f32 key column c (Key = KKK32: ORDER BY a, b, c; with kQKey2).
+constexpr int kQPred = 1, kQRank = 2, kQKey2 = 4, kQKey3 = 8;
 template <class Key, int Q>
 struct QCfg {
     static constexpr int kRowBytes = static_cast<int>(sizeof(Key)) +
-                                     ((Q & (kQRank | kQKey2)) ? 4 : 0) + ((Q & kQPred) ? 4 : 0);
+                                     ((Q & (kQRank | kQKey2)) ? 4 : 0) + ((Q & kQKey3) ? 4 : 0) +
+                                     ((Q & kQPred) ? 4 : 0);
     static constexpr int kItems =
         Q == 0 ? Cfg<Key>::kItems : (kRowBytes <= 8 ? 8 : 4);  // rows per consumer thread
     static constexpr int kTileKeys = Q == 0 ? Cfg<Key>::kTileKeys : kNC * kItems;
     static constexpr int kVecPerThread = kItems / KeyTraits<Key>::kVec;
     static constexpr int kOffB = kTileKeys * static_cast<int>(sizeof(Key));  // column b
-    static constexpr int kOffP = kOffB + ((Q & (kQRank | kQKey2)) ? kTileKeys * 4 : 0);  // pred
+    static constexpr int kOffC = kOffB + ((Q & (kQRank | kQKey2)) ? kTileKeys * 4 : 0);  // key 3
+    static constexpr int kOffP = kOffC + ((Q & kQKey3) ? kTileKeys * 4 : 0);  // predicate
     static_assert(Q == 0 || kTileKeys * kRowBytes <= kTileBytes, "stage size");
     static_assert(kTileKeys % 4 == 0, "TMA sizes are multiples of 16 bytes");
 };
@@ -128,6 +134,9 @@ struct SelectParams {
     const float* col_b;    // kQRank: column b of f = key + rank_w * b; kQKey2: second key
     float* out_keys2;      // kQKey2: b of each result row
     uint32_t order2_min;   // kQKey2: b ascending (1) or descending (0)
+    const float* col_c;    // kQKey3: third key column
+    float* out_keys3;
+    uint32_t order3_min;
     const uint32_t* pred;  // kQPred: predicate column
     float rank_w;
     uint32_t pred_in;      // 1: membership (pred < 64 and bit pred of pred_mask); 0: range
@@ -186,18 +195,42 @@ struct GBuf<E64> {
     }
 };
 
+template <>
+struct GBuf<E96> {
+    uint64_t* c;
+    uint32_t* c3;
+    uint32_t* ni;
+    __device__ __forceinline__ void init(unsigned char* base, size_t cap) {
+        c = reinterpret_cast<uint64_t*>(base);
+        c3 = reinterpret_cast<uint32_t*>(base + 8 * cap);
+        ni = reinterpret_cast<uint32_t*>(base + 12 * cap);
+    }
+    __device__ __forceinline__ E96 ld(size_t i) const {
+        return E96{__ldcg(c + i), __ldcg(c3 + i), __ldcg(ni + i)};
+    }
+    __device__ __forceinline__ void st(size_t i, E96 e) const {
+        __stcg(c + i, e.c);
+        __stcg(c3 + i, e.c3);
+        __stcg(ni + i, e.ni);
+    }
+};
+
 // Bounds as 64-bit words: E32 the packed entry (exact, index included); E64 the code
 // only, read back as {code, ni = 0} -- i.e. non-strict on that code (still valid).
 __device__ __forceinline__ unsigned long long bound_word(E32 e) { return e.v; }
 __device__ __forceinline__ unsigned long long bound_word(E64 e) { return e.c; }
+__device__ __forceinline__ unsigned long long bound_word(E96 e) { return e.c; }
 template <class E>
 __device__ __forceinline__ E from_bound_word(unsigned long long w);
 template <>
 __device__ __forceinline__ E32 from_bound_word<E32>(unsigned long long w) { return E32{w}; }
 template <>
 __device__ __forceinline__ E64 from_bound_word<E64>(unsigned long long w) { return E64{w, 0u}; }
+template <>
+__device__ __forceinline__ E96 from_bound_word<E96>(unsigned long long w) { return E96{w, 0u, 0u}; }
 __device__ __forceinline__ void tau_publish(WsHeader* h, E32 e) { atomicMax(&h->tau_g, e.v); }
 __device__ __forceinline__ void tau_publish(WsHeader* h, E64 e) { atomicMax(&h->tau_g, e.c); }
+__device__ __forceinline__ void tau_publish(WsHeader* h, E96 e) { atomicMax(&h->tau_g, e.c); }
 
 __device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -305,12 +338,21 @@ template <class Key>
 __device__ __forceinline__ E32 bound_get(const CtaState<E32, Key>& st) { return E32{st.tau_w}; }
 template <class Key>
 __device__ __forceinline__ E64 bound_get(const CtaState<E64, Key>& st) { return st.tau; }
+template <class Key>
+__device__ __forceinline__ E96 bound_get(const CtaState<E96, Key>& st) { return st.tau; }
 template <class Key, bool MIN>
 __device__ __forceinline__ void bound_set(CtaState<E32, Key>* st, E32 t) {
     if (t.v > st->tau_w) st->tau_w = t.v;
 }
 template <class Key, bool MIN>
 __device__ __forceinline__ void bound_set(CtaState<E64, Key>* st, E64 t) {
+    if (better(t, st->tau)) {
+        st->tau = t;
+        st->par = make_par<Key, MIN>(t);
+    }
+}
+template <class Key, bool MIN>
+__device__ __forceinline__ void bound_set(CtaState<E96, Key>* st, E96 t) {
     if (better(t, st->tau)) {
         st->tau = t;
         st->par = make_par<Key, MIN>(t);
@@ -323,6 +365,10 @@ __device__ __forceinline__ Par<E32, Key> load_par(const CtaState<E32, Key>& st) 
 }
 template <class Key, bool MIN>
 __device__ __forceinline__ Par<E64, Key> load_par(const CtaState<E64, Key>& st) {
+    return st.par;
+}
+template <class Key, bool MIN>
+__device__ __forceinline__ Par<E96, Key> load_par(const CtaState<E96, Key>& st) {
     return st.par;
 }
 
@@ -474,6 +520,10 @@ __device__ __forceinline__ unsigned long long code_word<E32>(uint32_t c) {
 }
 template <>
 __device__ __forceinline__ unsigned long long code_word<E64>(uint64_t c) {
+    return c;
+}
+template <>
+__device__ __forceinline__ unsigned long long code_word<E96>(uint64_t c) {
     return c;
 }
 
@@ -812,8 +862,10 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
         return static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
     };
     if constexpr ((Q & kQKey2) != 0) {
-        // compound key: 64-bit codes (code(a) << 32 | code2(b)); fast test on the code
+        // compound key: 64-bit codes (code(a) << 32 | code2(b)) [+ code3(c)]; fast test
+        // on the 64-bit code
         uint64_t cc[ITEMS];
+        uint32_t c3[ITEMS];
         const float4* sa = reinterpret_cast<const float4*>(slot_data);
         const float4* sb = reinterpret_cast<const float4*>(slot_data + QC::kOffB);
 #pragma unroll
@@ -823,6 +875,21 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
             for (int w = 0; w < VEC; ++w)
                 cc[j * VEC + w] = KT::template code2<MIN>(vget(a, w), vget(b, w), p.order2_min);
         }
+        if constexpr ((Q & kQKey3) != 0) {
+            const float4* sc = reinterpret_cast<const float4*>(slot_data + QC::kOffC);
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+                const float4 cv = sc[tid + j * kNC];
+#pragma unroll
+                for (int w = 0; w < VEC; ++w) c3[j * VEC + w] = KT::code3(vget(cv, w), p.order3_min);
+            }
+        }
+        auto mk = [&](int q) -> E {
+            if constexpr ((Q & kQKey3) != 0)
+                return E::make(cc[q], c3[q], lbase + pos_of(q));
+            else
+                return E::make(cc[q], lbase + pos_of(q));
+        };
         uint32_t mask = (ITEMS >= 32) ? 0xFFFFFFFFu : ((1u << ITEMS) - 1u);
         if constexpr ((Q & kQPred) != 0) {
             const uint4* sp = reinterpret_cast<const uint4*>(slot_data + QC::kOffP);
@@ -856,12 +923,11 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
             if (!__any_sync(0xFFFFFFFFu, mask != 0u)) return 0;
 #pragma unroll
             for (int q = 0; q < ITEMS; ++q)
-                if (((mask >> q) & 1u) && !better(E::make(cc[q], lbase + pos_of(q)), pr.tau))
-                    mask &= ~(1u << q);
+                if (((mask >> q) & 1u) && !better(mk(q), pr.tau)) mask &= ~(1u << q);
         }
         E ents[ITEMS];
 #pragma unroll
-        for (int q = 0; q < ITEMS; ++q) ents[q] = E::make(cc[q], lbase + pos_of(q));
+        for (int q = 0; q < ITEMS; ++q) ents[q] = mk(q);
         return append<E, ITEMS>(buf, s_cnt, ents, mask, limit);
     } else {
     Key x[ITEMS];
@@ -960,7 +1026,10 @@ template <class Key, bool MIN, int Q>
 __device__ __forceinline__ typename KeyTraits<Key>::E query_entry(const SelectParams& p,
                                                                   const Key* keys, uint64_t row) {
     using KT = KeyTraits<Key>;
-    if constexpr ((Q & kQKey2) != 0)
+    if constexpr ((Q & kQKey3) != 0)
+        return KT::E::make(KT::template code2<MIN>(keys[row].a, p.col_b[row], p.order2_min),
+                           KT::code3(p.col_c[row], p.order3_min), static_cast<uint32_t>(row));
+    else if constexpr ((Q & kQKey2) != 0)
         return KT::E::make(KT::template code2<MIN>(keys[row].a, p.col_b[row], p.order2_min),
                            static_cast<uint32_t>(row));
     else
@@ -1103,6 +1172,11 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             if constexpr ((Q & (kQRank | kQKey2)) != 0) {  // one slab per column (head == 0)
                 tma_load_1d(dst + QCfg<Key, Q>::kOffB, p.col_b + lo,
                             static_cast<uint32_t>(len * 4), &full[slot], policy);
+                bytes += static_cast<uint32_t>(len * 4);
+            }
+            if constexpr ((Q & kQKey3) != 0) {
+                tma_load_1d(dst + QCfg<Key, Q>::kOffC, p.col_c + lo, static_cast<uint32_t>(len * 4),
+                            &full[slot], policy);
                 bytes += static_cast<uint32_t>(len * 4);
             }
             if constexpr ((Q & kQPred) != 0) {
@@ -1329,6 +1403,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = Key{0};
             if constexpr ((Q & kQKey2) != 0)
                 if (p.out_keys2) p.out_keys2[j] = 0.f;
+            if constexpr ((Q & kQKey3) != 0)
+                if (p.out_keys3) p.out_keys3[j] = 0.f;
             if (p.out_payload) p.out_payload[j] = 0u;
             continue;
         }
@@ -1337,6 +1413,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if constexpr ((Q & kQKey2) != 0) {
             if (p.out_keys) static_cast<float*>(p.out_keys)[j] = keys[row].a;
             if (p.out_keys2) p.out_keys2[j] = p.col_b[row];
+            if constexpr ((Q & kQKey3) != 0)
+                if (p.out_keys3) p.out_keys3[j] = p.col_c[row];
         } else {
             if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = query_key<Key, Q>(p, keys, row);
         }

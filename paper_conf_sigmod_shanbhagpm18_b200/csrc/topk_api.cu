@@ -45,7 +45,9 @@ bool device_info(int* sms, int* major) {
 }
 
 size_t key_size(topk_dtype_t dt) { return dt == TOPK_F64 ? 8 : 4; }
-size_t entry_bytes(topk_dtype_t dt) { return dt == TOPK_F64 ? 12 : 8; }
+// workspace candidate entry bytes: 8 (32-bit codes); 12 for f64 / two compound keys,
+// 16 for three compound keys (E96) -- the 64-bit layouts share the larger size
+size_t entry_bytes(topk_dtype_t dt) { return dt == TOPK_F64 ? 16 : 8; }
 
 uint32_t next_pow2_u32(uint32_t x) {
     uint32_t p = 1;
@@ -119,6 +121,10 @@ uint32_t query_tile_keys(topk_dtype_t dt, int q) {
     using topk::kQPred;
     using topk::kQRank;
     using topk::kQKey2;
+    using topk::kQKey3;
+    if (q & kQKey3)
+        return (q & kQPred) ? QCfg<topk::KKK32, kQKey2 | kQKey3 | kQPred>::kTileKeys
+                            : QCfg<topk::KKK32, kQKey2 | kQKey3>::kTileKeys;
     if (q & kQKey2)
         return (q & kQPred) ? QCfg<topk::KK32, kQKey2 | kQPred>::kTileKeys
                             : QCfg<topk::KK32, kQKey2>::kTileKeys;
@@ -195,6 +201,9 @@ struct QueryArgs {
     topk_pred_t pred{};
     float* out_keys2 = nullptr;  // kQKey2
     uint32_t order2_min = 0;
+    const float* col_c = nullptr;  // kQKey3
+    float* out_keys3 = nullptr;
+    uint32_t order3_min = 0;
 };
 
 static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint32_t* payload,
@@ -284,7 +293,11 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
     if (qa.q & topk::kQKey2) {
         p.out_keys2 = qa.out_keys2;
         p.order2_min = qa.order2_min;
-        return launch_variant(topk::kKeyKK, mn, true, qa.q, p, grid, st) == cudaSuccess
+        p.col_c = qa.col_c;
+        p.out_keys3 = qa.out_keys3;
+        p.order3_min = qa.order3_min;
+        return launch_variant((qa.q & topk::kQKey3) ? topk::kKeyKKK : topk::kKeyKK, mn, true, qa.q,
+                              p, grid, st) == cudaSuccess
                    ? TOPK_OK : TOPK_ERR_CUDA;
     }
     return launch_variant(key_kind(dtype), mn, qa.q ? true : filt, qa.q, p, grid, st) == cudaSuccess
@@ -449,6 +462,37 @@ topk_status_t topk_radix(topk_dtype_t dtype, const void* keys, uint64_t n, uint3
     if (e != cudaSuccess) return TOPK_ERR_CUDA;
     g_launches.fetch_add(static_cast<uint64_t>(launches), std::memory_order_relaxed);
     return TOPK_OK;
+}
+
+topk_status_t topk_kkk(const float* keys1, const float* keys2, const float* keys3,
+                       const topk_pred_t* pred, const uint32_t* payload, uint64_t n, uint32_t k,
+                       topk_order_t order1, topk_order_t order2, topk_order_t order3,
+                       float* out_keys1, float* out_keys2, float* out_keys3,
+                       uint32_t* out_payload, int64_t* out_idx, void* ws, size_t ws_bytes,
+                       void* stream) {
+    if (!keys1 || !keys2 || !keys3 || n == 0 || n > kMaxLaunchN) return TOPK_ERR_INVALID_ARG;
+    if (!valid_order(order1) || !valid_order(order2) || !valid_order(order3))
+        return TOPK_ERR_INVALID_ARG;
+    QueryArgs qa;
+    qa.q = topk::kQKey2 | topk::kQKey3;
+    qa.rank_b = keys2;
+    qa.out_keys2 = out_keys2;
+    qa.order2_min = order2 == TOPK_SMALLEST ? 1u : 0u;
+    qa.col_c = keys3;
+    qa.out_keys3 = out_keys3;
+    qa.order3_min = order3 == TOPK_SMALLEST ? 1u : 0u;
+    if (pred) {
+        if ((pred->kind != TOPK_PRED_RANGE && pred->kind != TOPK_PRED_IN) || !pred->col)
+            return TOPK_ERR_INVALID_ARG;
+        qa.q |= topk::kQPred;
+        qa.pred = *pred;
+    }
+    auto misaligned = [](const void* c) { return reinterpret_cast<uintptr_t>(c) % 16 != 0; };
+    if (misaligned(keys1) || misaligned(keys2) || misaligned(keys3) ||
+        (pred && misaligned(pred->col)) || (payload && misaligned(payload)))
+        return TOPK_ERR_INVALID_ARG;
+    return select_one(TOPK_F64, keys1, payload, n, 0, k, order1, TOPK_MODE_FILTER, out_keys1,
+                      out_payload, out_idx, ws, ws_bytes, stream, qa);
 }
 
 topk_status_t topk_f32(const float* keys, uint64_t n, uint32_t k, topk_order_t order,

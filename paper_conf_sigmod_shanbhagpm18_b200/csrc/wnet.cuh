@@ -44,6 +44,15 @@ __device__ __forceinline__ E64 shfl_xor_e<E64>(const E64& e, int m) {
     return E64{(static_cast<uint64_t>(hi) << 32) | lo, ni};
 }
 
+template <>
+__device__ __forceinline__ E96 shfl_xor_e<E96>(const E96& e, int m) {
+    const uint32_t lo = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.c), m);
+    const uint32_t hi = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.c >> 32), m);
+    const uint32_t c3 = __shfl_xor_sync(0xFFFFFFFFu, e.c3, m);
+    const uint32_t ni = __shfl_xor_sync(0xFFFFFFFFu, e.ni, m);
+    return E96{(static_cast<uint64_t>(hi) << 32) | lo, c3, ni};
+}
+
 // Compare-exchange of two registers: afterwards a holds the better entry iff a_better.
 template <class E>
 __device__ __forceinline__ void cmpx(E& a, E& b, bool a_better) {

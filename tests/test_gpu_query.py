@@ -218,3 +218,50 @@ def test_compound_keys_predicate_payload(cuda_device, dist):
     pay = datagen.payload(N, seed=330)
     run_kk(k1, k2, 64, True, True, pred=("range", col, 10, 60), payload=pay)
     run_kk(k1, k2, 64, False, True, pred=("in", col, (1 << 7) | (1 << 40)), payload=pay)
+
+
+# ---- three compound keys: ORDER BY k1, k2, k3 LIMIT k (KKKV) ----
+
+def run_kkk(cols, k, orders=(True, True, True), pred=None, payload=None):
+    dev = "cuda"
+    gpred = None if pred is None else (pred[0], pred[1].to(dev), *pred[2:])
+    out = tk.topk_kkk(*[c.to(dev) for c in cols], k, orders, pred=gpred,
+                      payload=None if payload is None else payload.to(dev))
+    torch.cuda.synchronize()
+    h = [host(c) for c in cols]
+    oi = np.full(k, -1, dtype=np.int64)
+    ov = [np.zeros(k, dtype=np.float32) for _ in range(3)]
+    rows = np.arange(h[0].shape[0])
+    if pred is not None:  # the plain plan: filter, then the compound top-k
+        c = host(pred[1])
+        rows = np.nonzero((c >= pred[2]) & (c < pred[3]))[0]
+    m = min(k, rows.shape[0])
+    if m:
+        r = oracle.topk_kkk(*[x[rows] for x in h], m, orders)
+        oi[:m] = rows[r[3]]
+        for j in range(3):
+            ov[j][:m] = r[j]
+    gi = out[3].cpu().numpy()
+    assert np.array_equal(gi, oi), f"indices differ: first at {np.nonzero(gi != oi)[0][:5]}"
+    for j in range(3):
+        assert host(out[j]).tobytes() == ov[j].tobytes()
+    if payload is not None:
+        ph = host(payload)
+        assert np.array_equal(host(out[4]), np.where(oi >= 0, ph[np.maximum(oi, 0)], 0).astype(np.uint32))
+
+
+@pytest.mark.parametrize("orders", [(True, True, True), (False, True, False), (True, False, True)])
+def test_three_keys(cuda_device, orders):
+    cols = [datagen.generate("fewdistinct", N, "f32", seed=331),
+            datagen.generate("fewdistinct", N, "f32", seed=332),
+            datagen.generate("uniform", N, "f32", seed=333)]
+    for k in (1, 64, 256, 2048):
+        run_kkk(cols, k, orders)
+
+
+def test_three_keys_full_ties_predicate_payload(cuda_device):
+    cols = [datagen.generate("fewdistinct", N, "f32", seed=334) for _ in range(3)]
+    run_kkk(cols, 500, (True, True, False))  # 16^3 distinct tuples: the row id decides
+    col = u32col(N, 335, 10)
+    pay = datagen.payload(N, seed=336)
+    run_kkk(cols, 64, (False, False, True), pred=("range", col, 3, 8), payload=pay)
