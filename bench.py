@@ -333,7 +333,12 @@ def run_ours(args):
         cfgs.append({"config": "f3 KKV: 2^28 rows, ORDER BY k1 DESC, k2 DESC LIMIT 64, u32 value",
                      "us": round(t * 1e3, 1), "rows_per_s": n4 / (t / 1e3),
                      "frac_hbm": n4 * 8 / (t / 1e3) / 1e9 / peaks()[0]})
-        del k1, k2, pv, a, b
+        k3 = datagen.generate("uniform", n4, "f32", seed=datagen.config_seed(7, 2), device=dev)
+        t = timed(lambda: tk.topk_kkk(k1, k2, k3, 64, payload=pv))
+        cfgs.append({"config": "f3 KKKV: 2^28 rows, ORDER BY k1, k2, k3 DESC LIMIT 64, u32 value",
+                     "us": round(t * 1e3, 1), "rows_per_s": n4 / (t / 1e3),
+                     "frac_hbm": n4 * 12 / (t / 1e3) / 1e9 / peaks()[0]})
+        del k1, k2, k3, pv, a, b
         for kk in (32, 256):
             t = timed(lambda: tk.topk(x, kk, True, mode="pure"), 2)
             cfgs.append({"config": f"pure mode (paper's data-independent network on every key), "

@@ -910,9 +910,10 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
         }
         if (pr.active) {
             // superset test on the code (>= always valid; > once every row of the tile
-            // comes after the bound's row), then the exact (code, row) test
+            // comes after the bound's row -- only when the 64-bit code is the whole key:
+            // with a third key an equal code may still win on c3), then the exact test
             const uint64_t tc = pr.tau.c;
-            const bool strict = lbase > pr.strict_after;
+            const bool strict = (Q & kQKey3) == 0 && lbase > pr.strict_after;
             uint32_t keep = 0;
 #pragma unroll
             for (int q = 0; q < ITEMS; ++q) {
