@@ -1,6 +1,6 @@
 """Run one hot-path op a few times (for an ncu capture of its kernel; dev tool).
 
-    python tools/prof_any.py select|query1|query2|kk|radix K
+    python tools/prof_any.py select|query1|query2|kk|kkk|radix K
 """
 import os
 import sys
@@ -31,6 +31,11 @@ elif op == "kk":
     k1 = datagen.generate("uniform", n, "f32", seed=datagen.config_seed(7), device=dev)
     k2 = datagen.generate("uniform", n, "f32", seed=datagen.config_seed(7, 1), device=dev)
     f = lambda: tk.topk_kk(k1, k2, k)
+elif op == "kkk":
+    n = 1 << 28
+    ks = [datagen.generate("uniform", n, "f32", seed=datagen.config_seed(7, j), device=dev)
+          for j in range(3)]
+    f = lambda: tk.topk_kkk(*ks, k)
 else:
     raise SystemExit(f"unknown op {op}")
 for _ in range(4):
