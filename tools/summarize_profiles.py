@@ -124,13 +124,19 @@ def main(rnd):
         agg = defaultdict(list)
         for r in rows[1:]:
             try:
-                agg[re.sub(r"\(.*", "", r[ki])].append(float(r[vi].replace(",", "")))
+                name = re.sub(r"\(.*", "", r[ki])
+                v = float(r[vi].replace(",", ""))
+                if "select_kernel" in name:  # the timed step vs the e2e leg's 2^26-key chunks
+                    name += " [2^29-key step]" if v > 150e3 else " [e2e: 2^26-key chunk]"
+                agg[name].append(v)
             except ValueError:
                 pass
         tot = sum(sum(v) for v in agg.values())
         lines = [f"# Launch list of `bench.py --steps 20 --warmup 3` ({rnd})", "",
                  "`ncu --metrics gpu__time_duration.sum --clock-control none -k regex:'select_kernel|merge_kernel' -c 60` "
-                 "(only this library's kernels; per-launch times are cold-cache and serialised).",
+                 "(only this library's kernels; per-launch times are cold-cache and serialised). "
+                 "The timed step (N=1) is exactly one select_kernel launch over 2^29 keys (share of "
+                 "the step: 1.0); the e2e leg adds one launch per 2^26-key host chunk + one merge.",
                  "", "| kernel | launches | mean us | share of our kernel time |", "|---|---|---|---|"]
         for name, v in sorted(agg.items(), key=lambda kv: -sum(kv[1])):
             lines.append(f"| {name} | {len(v)} | {sum(v) / len(v) / 1e3:.1f} | {sum(v) / tot:.3f} |")
