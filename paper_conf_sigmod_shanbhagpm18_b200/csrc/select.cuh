@@ -459,23 +459,28 @@ template <class E, class Key>
 __device__ void rank_rows(CtaState<E, Key>* st, const Ctx& cx) {
     if (threadIdx.x < kPubRows) st->best[threadIdx.x] = 0ull;
     CSync::sync();
+    // one warp per sample: the lanes count over the row, a warp reduction sums
     const int RG = cx.nrows * cx.G;
-    for (int q = threadIdx.x; q < RG; q += kNC) {
+    const int lane = threadIdx.x & 31;
+    for (int q = threadIdx.x >> 5; q < RG; q += kNC / 32) {
         const int r = q / cx.G;
         const int ji = cx.j_lo + r;
         const int t = (cx.k + (1 << ji) - 1) >> ji;
         const unsigned long long v = cx.scratch[q];
-        if (v == 0ull) continue;
+        if (v == 0ull) continue;  // warp-uniform
         const unsigned long long* row = cx.scratch + r * cx.G;
-        int gt = 0, ge = 0;
-#pragma unroll 4
-        for (int c2 = 0; c2 < cx.G; ++c2) {
-            gt += row[c2] > v ? 1 : 0;
-            ge += row[c2] >= v ? 1 : 0;
+        unsigned gt = 0, ge = 0;
+        for (int c2 = lane; c2 < cx.G; c2 += 32) {
+            const unsigned long long x = row[c2];
+            gt += x > v ? 1u : 0u;
+            ge += x >= v ? 1u : 0u;
         }
+        gt = __reduce_add_sync(0xFFFFFFFFu, gt);
+        ge = __reduce_add_sync(0xFFFFFFFFu, ge);
         // v is the t-th largest (code-only samples of different CTAs may be equal words:
-        // every thread holding that value writes the same word)
-        if (gt <= t - 1 && t - 1 < ge) st->best[ji] = v;
+        // every warp holding that value writes the same word)
+        if (lane == 0 && static_cast<int>(gt) <= t - 1 && t - 1 < static_cast<int>(ge))
+            st->best[ji] = v;
     }
     CSync::sync();
 }
