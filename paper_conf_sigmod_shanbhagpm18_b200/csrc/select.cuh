@@ -445,7 +445,7 @@ struct Ctx {
     int k, K;
     int G, gmax, J;
     int j_lo, nrows;  // rank-bound rows used: j_lo .. j_lo + nrows - 1 (t <= G)
-    int Lp;           // code network size log2 K' (K' = max(K, 16)); -1: not used (K > 512)
+    int Lp;           // code network size log2 K' (K' = min(max(K, 16), 512)); -1: not used
     void* codes;      // shared: code-network scratch (8 x K' codes)
     bool filter;
 };
@@ -459,28 +459,23 @@ template <class E, class Key>
 __device__ void rank_rows(CtaState<E, Key>* st, const Ctx& cx) {
     if (threadIdx.x < kPubRows) st->best[threadIdx.x] = 0ull;
     CSync::sync();
-    // one warp per sample: the lanes count over the row, a warp reduction sums
     const int RG = cx.nrows * cx.G;
-    const int lane = threadIdx.x & 31;
-    for (int q = threadIdx.x >> 5; q < RG; q += kNC / 32) {
+    for (int q = threadIdx.x; q < RG; q += kNC) {
         const int r = q / cx.G;
         const int ji = cx.j_lo + r;
         const int t = (cx.k + (1 << ji) - 1) >> ji;
         const unsigned long long v = cx.scratch[q];
-        if (v == 0ull) continue;  // warp-uniform
+        if (v == 0ull) continue;
         const unsigned long long* row = cx.scratch + r * cx.G;
-        unsigned gt = 0, ge = 0;
-        for (int c2 = lane; c2 < cx.G; c2 += 32) {
-            const unsigned long long x = row[c2];
-            gt += x > v ? 1u : 0u;
-            ge += x >= v ? 1u : 0u;
+        int gt = 0, ge = 0;
+#pragma unroll 4
+        for (int c2 = 0; c2 < cx.G; ++c2) {
+            gt += row[c2] > v ? 1 : 0;
+            ge += row[c2] >= v ? 1 : 0;
         }
-        gt = __reduce_add_sync(0xFFFFFFFFu, gt);
-        ge = __reduce_add_sync(0xFFFFFFFFu, ge);
         // v is the t-th largest (code-only samples of different CTAs may be equal words:
-        // every warp holding that value writes the same word)
-        if (lane == 0 && static_cast<int>(gt) <= t - 1 && t - 1 < static_cast<int>(ge))
-            st->best[ji] = v;
+        // every thread holding that value writes the same word)
+        if (gt <= t - 1 && t - 1 < ge) st->best[ji] = v;
     }
     CSync::sync();
 }
@@ -630,7 +625,7 @@ __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
 }
 
 // Collective flush (consumers) of the candidate bag buf[0 .. cnt):
-//   code path (filter mode, K <= 512; every stream flush, and a final flush of a large
+//   code path (filter mode, ranking min(K, 512) codes; every stream flush, and a final flush of a large
 //     bag): the code-only network (cnet.cuh) gives the bag's k-th best code and its
 //     2^j-th best codes -> publish, bound round, drop every entry worse than the new
 //     bound.  A stream flush ends here unless ties kept the bag over half full.
@@ -655,21 +650,23 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
     bool done = false;
     // (tie-heavy input -- a code bound cannot separate equal codes -- makes the code
     // path useless: after it failed once, stream flushes go straight to the exact path)
-    const bool try_code = !st->ties && (publish || cnt > 2 * K);
+    const bool try_code = !st->ties && (publish || (cnt > 2 * K && K <= (1 << cx.Lp)));
     bool tried = false;
     if (cx.filter && cx.Lp >= 0 && !(c_dbg & 1) && try_code) {
         tried = true;
         C* S = static_cast<C*>(cx.codes);
         cnet_topk_codes<E, kNC / 32, CSync>(buf, cnt, cx.Lp, S, w, lane);
-        if (publish && threadIdx.x < cx.J && cnt >= (1 << threadIdx.x)) {
+        const int Kp = 1 << cx.Lp;  // codes the network ranked (S[0 .. Kp))
+        if (publish && threadIdx.x < cx.J && threadIdx.x <= cx.Lp && cnt >= (1 << threadIdx.x)) {
             st_relaxed_u64(cx.pub + static_cast<size_t>(threadIdx.x) * cx.gmax + c,
                            code_word<E>(S[(1 << threadIdx.x) - 1]));
             __threadfence();
         }
-        const E own = cnt >= k ? from_bound_word<E>(code_word<E>(S[k - 1])) : E::sentinel();
+        // the bag's own k-th best code (only if the network ranked that far)
+        const E own =
+            (cnt >= k && k <= Kp) ? from_bound_word<E>(code_word<E>(S[k - 1])) : E::sentinel();
         // half of the top K' codes equal: heavy ties (few distinct keys), which a code
         // bound cannot separate -- finish exactly (strict (code, index) bound) at once
-        const int Kp = 1 << cx.Lp;
         const bool heavy = cnt >= Kp && S[Kp - 1] == S[Kp / 2 - 1];
         take_bounds<Key, MIN>(st, cx, own, publish);
         if (!heavy) cnt = compact_bag<E>(buf, cnt, bound_get(*st), st->wcnt);
@@ -867,18 +864,58 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
         return static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
     };
     if constexpr ((Q & kQKey2) != 0) {
-        // compound key: 64-bit codes (code(a) << 32 | code2(b)) [+ code3(c)]; fast test
-        // on the 64-bit code
+        // compound key: 64-bit codes (code(a) << 32 | code2(b)) [+ code3(c)].  The
+        // streamed test is one float compare of the first key against the bound's first
+        // key (non-strict: a superset of "may beat the bound"); only warps with a passing
+        // row read the other columns and build codes for the exact entry test.
+        float av[ITEMS];
+        {
+            const float4* sa = reinterpret_cast<const float4*>(slot_data);
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+                const float4 a = sa[tid + j * kNC];
+#pragma unroll
+                for (int w = 0; w < VEC; ++w) av[j * VEC + w] = vget(a, w);
+            }
+        }
+        uint32_t mask = (ITEMS >= 32) ? 0xFFFFFFFFu : ((1u << ITEMS) - 1u);
+        if (tlen < static_cast<uint32_t>(TK)) {
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                if (pos_of(q) >= tlen) mask &= ~(1u << q);
+        }
+        if (pr.active) {
+            const float t1 = KeyTraits<float>::template decode<MIN>(pr.tau.c >> 32);
+            uint32_t f = 0;
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                f |= static_cast<uint32_t>(KeyTraits<float>::template fast<MIN, false>(av[q], t1)) << q;
+            mask &= f;
+            if (!__any_sync(0xFFFFFFFFu, mask != 0u)) return 0;
+        }
+        if constexpr ((Q & kQPred) != 0) {
+            const uint4* sp = reinterpret_cast<const uint4*>(slot_data + QC::kOffP);
+            uint32_t pm = 0;
+#pragma unroll
+            for (int j = 0; j < VPT; ++j) {
+                const uint4 u = sp[tid + j * kNC];
+#pragma unroll
+                for (int w = 0; w < VEC; ++w)
+                    pm |= static_cast<uint32_t>(pred_ok(p, vget(u, w))) << (j * VEC + w);
+            }
+            mask &= pm;
+        }
         uint64_t cc[ITEMS];
         uint32_t c3[ITEMS];
-        const float4* sa = reinterpret_cast<const float4*>(slot_data);
-        const float4* sb = reinterpret_cast<const float4*>(slot_data + QC::kOffB);
+        {
+            const float4* sb = reinterpret_cast<const float4*>(slot_data + QC::kOffB);
 #pragma unroll
-        for (int j = 0; j < VPT; ++j) {
-            const float4 a = sa[tid + j * kNC], b = sb[tid + j * kNC];
+            for (int j = 0; j < VPT; ++j) {
+                const float4 b = sb[tid + j * kNC];
 #pragma unroll
-            for (int w = 0; w < VEC; ++w)
-                cc[j * VEC + w] = KT::template code2<MIN>(vget(a, w), vget(b, w), p.order2_min);
+                for (int w = 0; w < VEC; ++w)
+                    cc[j * VEC + w] = KT::template code2<MIN>(av[j * VEC + w], vget(b, w), p.order2_min);
+            }
         }
         if constexpr ((Q & kQKey3) != 0) {
             const float4* sc = reinterpret_cast<const float4*>(slot_data + QC::kOffC);
@@ -895,38 +932,7 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
             else
                 return E::make(cc[q], lbase + pos_of(q));
         };
-        uint32_t mask = (ITEMS >= 32) ? 0xFFFFFFFFu : ((1u << ITEMS) - 1u);
-        if constexpr ((Q & kQPred) != 0) {
-            const uint4* sp = reinterpret_cast<const uint4*>(slot_data + QC::kOffP);
-            uint32_t pm = 0;
-#pragma unroll
-            for (int j = 0; j < VPT; ++j) {
-                const uint4 u = sp[tid + j * kNC];
-#pragma unroll
-                for (int w = 0; w < VEC; ++w)
-                    pm |= static_cast<uint32_t>(pred_ok(p, vget(u, w))) << (j * VEC + w);
-            }
-            mask &= pm;
-        }
-        if (tlen < static_cast<uint32_t>(TK)) {
-#pragma unroll
-            for (int q = 0; q < ITEMS; ++q)
-                if (pos_of(q) >= tlen) mask &= ~(1u << q);
-        }
-        if (pr.active) {
-            // superset test on the code (>= always valid; > once every row of the tile
-            // comes after the bound's row -- only when the 64-bit code is the whole key:
-            // with a third key an equal code may still win on c3), then the exact test
-            const uint64_t tc = pr.tau.c;
-            const bool strict = (Q & kQKey3) == 0 && lbase > pr.strict_after;
-            uint32_t keep = 0;
-#pragma unroll
-            for (int q = 0; q < ITEMS; ++q) {
-                const bool f = strict ? cc[q] > tc : cc[q] >= tc;
-                keep |= static_cast<uint32_t>(f) << q;
-            }
-            mask &= keep;
-            if (!__any_sync(0xFFFFFFFFu, mask != 0u)) return 0;
+        if (pr.active) {  // exact entry test (lexicographic codes, then the row)
 #pragma unroll
             for (int q = 0; q < ITEMS; ++q)
                 if (((mask >> q) & 1u) && !better(mk(q), pr.tau)) mask &= ~(1u << q);
@@ -1088,7 +1094,9 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         cx.nrows = cx.J - cx.j_lo < maxrows ? cx.J - cx.j_lo : maxrows;
     }
     cx.filter = FILTER;
-    cx.Lp = (FILTER && K <= 512) ? (K < 16 ? 4 : __ffs(K) - 1) : -1;
+    // K > 512: the code network still gives the bag's 2^j-th best codes for j <= 9,
+    // whose cross-CTA rank bound bounds the global k-th best (t = ceil(k / 2^j) <= G)
+    cx.Lp = FILTER ? (K < 16 ? 4 : min(__ffs(K) - 1, 9)) : -1;
     cx.codes = scratch + kScratch;
 
     if (tid == 0) {
