@@ -265,7 +265,9 @@ def run_ours(args):
             rv.append({"k": kk, "radix_us": round(t * 1e3, 1), "bitonic_us": tb,
                        "model_radix_us": round(cm.radix_time(n, KEY_BYTES, hw) * 1e6, 1),
                        "model_bitonic_paper_us": round(cm.bitonic_time(n, KEY_BYTES, kk, hw) * 1e6, 1),
-                       "model_choice": cm.choose(n, KEY_BYTES, kk, hw),
+                       "model_bitonic_b200_us": round(cm.bitonic_b200_time(n, KEY_BYTES, hw) * 1e6, 1),
+                       "model_choice_paper": cm.choose(n, KEY_BYTES, kk, hw),
+                       "model_choice_b200": cm.choose_b200(n, KEY_BYTES, kk, hw),
                        "measured_choice": "bitonic" if tb <= t * 1e3 else "radix"})
         extra["radix_vs_bitonic"] = rv
         adv = []

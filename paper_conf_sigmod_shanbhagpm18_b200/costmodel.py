@@ -77,5 +77,18 @@ def bitonic_time(n: int, w: int, k: int, hw: Hardware, x: int = 8) -> float:
 
 
 def choose(n: int, w: int, k: int, hw: Hardware) -> str:
-    """Model-based dispatch: the method with the smaller predicted time."""
+    """Model-based dispatch (the paper's models): the smaller predicted time."""
     return "bitonic" if bitonic_time(n, w, k, hw) <= radix_time(n, w, hw) else "radix"
+
+
+def bitonic_b200_time(n: int, w: int, hw: Hardware) -> float:
+    """This repo's B200 pass: every key read from HBM once, the network
+    run on the buffer filler's survivors only (~0.1 % of the keys on uniform data), the
+    intermediate runs on chip / in L2 -- bounded below by T_g's first term, D / B_G.
+    The paper's T_k (every key through shared memory) no longer applies."""
+    return n * w / hw.b_g
+
+
+def choose_b200(n: int, w: int, k: int, hw: Hardware) -> str:
+    """Dispatch with the B200 bitonic model against the paper's radix model."""
+    return "bitonic" if bitonic_b200_time(n, w, hw) <= radix_time(n, w, hw) else "radix"

@@ -54,3 +54,11 @@ def test_crossover_direction():
     hb = cm.b200(6563.0)
     assert hb.b_s == pytest.approx(148 * 128 * 1.965e9)
     assert math.isfinite(cm.radix_time(N, W, hb))
+
+
+def test_b200_model_prefers_one_pass():
+    """One read of the input (the B200 pass) beats radix's >= 2 reads at any k."""
+    hb = cm.b200(6563.0)
+    assert cm.bitonic_b200_time(N, W, hb) == pytest.approx(N * W / hb.b_g)
+    for k in (1, 32, 256, 1024, 2048):
+        assert cm.choose_b200(N, W, k, hb) == "bitonic"
