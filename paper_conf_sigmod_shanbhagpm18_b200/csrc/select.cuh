@@ -98,6 +98,14 @@ struct QCfg {
     static constexpr int kOffC = kOffB + ((Q & (kQRank | kQKey2)) ? kTileKeys * 4 : 0);  // key 3
     static constexpr int kOffP = kOffC + ((Q & kQKey3) ? kTileKeys * 4 : 0);  // predicate
     static_assert(Q == 0 || kTileKeys * kRowBytes <= kTileBytes, "stage size");
+    // ring: a query stage is TK rows of every column (<= one plain stage), so the ring
+    // budget of the plain form holds more of them (up to kStagesMax)
+    static constexpr int kSlotBytes = Q == 0 ? kTileBytes : (kTileKeys * kRowBytes + 127) / 128 * 128;
+    static constexpr int kStages =
+        Q == 0 ? Cfg<Key>::kStages
+               : (Cfg<Key>::kStages * kTileBytes / kSlotBytes < kStagesMax
+                      ? Cfg<Key>::kStages * kTileBytes / kSlotBytes
+                      : kStagesMax);
     static_assert(kTileKeys % 4 == 0, "TMA sizes are multiples of 16 bytes");
 };
 
@@ -1056,7 +1064,9 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     using E = typename KT::E;
     using C = Cfg<Key>;
     constexpr int TK = QCfg<Key, Q>::kTileKeys;
-    constexpr int kStages = C::kStages;
+    using QC = QCfg<Key, Q>;
+    constexpr int kStages = QC::kStages;
+    constexpr int kSlot = QC::kSlotBytes;
     static_assert(Q == 0 || FILTER, "query forms run in filter mode");
 
     extern __shared__ __align__(128) unsigned char smem[];
@@ -1064,8 +1074,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
 
     unsigned char* ring = smem;
     SBuf<E> buf;
-    buf.init(smem + static_cast<size_t>(kStages) * kTileBytes, kCap);
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + static_cast<size_t>(kStages) * kTileBytes +
+    buf.init(smem + static_cast<size_t>(kStages) * kSlot, kCap);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + static_cast<size_t>(kStages) * kSlot +
                                                  static_cast<size_t>(kCap) * SBuf<E>::kBytes);
     uint64_t* empty = full + kStages;
     unsigned long long* scratch = reinterpret_cast<unsigned long long*>(empty + kStages);
@@ -1186,7 +1196,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             const uint64_t lo = static_cast<uint64_t>(tile) * TK;
             const uint64_t len = min(static_cast<uint64_t>(TK), p.body_n - lo);
             uint32_t bytes = static_cast<uint32_t>(len * sizeof(Key));
-            unsigned char* dst = ring + static_cast<size_t>(slot) * kTileBytes;
+            unsigned char* dst = ring + static_cast<size_t>(slot) * kSlot;
             tma_load_1d(dst, body + lo, bytes, &full[slot], policy);
             if constexpr ((Q & (kQRank | kQKey2)) != 0) {  // one slab per column (head == 0)
                 tma_load_1d(dst + QCfg<Key, Q>::kOffB, p.col_b + lo,
@@ -1237,7 +1247,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         const uint64_t tlo = static_cast<uint64_t>(tile) * TK;
         const uint32_t tlen = static_cast<uint32_t>(min(static_cast<uint64_t>(TK), p.body_n - tlo));
         const uint32_t lbase = static_cast<uint32_t>(p.head + tlo);
-        const unsigned char* data = ring + static_cast<size_t>(slot) * kTileBytes;
+        const unsigned char* data = ring + static_cast<size_t>(slot) * kSlot;
         Par<E, Key> pr = load_par<Key, MIN>(st);
         auto consume = [&]() -> int {
             if constexpr (Q == 0)
@@ -1451,11 +1461,11 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     }
 }
 
-template <class Key>
+template <class Key, int Q = 0>
 constexpr size_t select_smem_bytes() {
-    return static_cast<size_t>(Cfg<Key>::kStages) * kTileBytes +
+    return static_cast<size_t>(QCfg<Key, Q>::kStages) * QCfg<Key, Q>::kSlotBytes +
            static_cast<size_t>(kCap) * SBuf<typename KeyTraits<Key>::E>::kBytes +
-           static_cast<size_t>(2 * Cfg<Key>::kStages) * 8 + static_cast<size_t>(kScratch) * 8 +
+           static_cast<size_t>(2 * QCfg<Key, Q>::kStages) * 8 + static_cast<size_t>(kScratch) * 8 +
            static_cast<size_t>(kCap / 512) * 512 *
                sizeof(typename CodeOf<typename KeyTraits<Key>::E>::C);  // code network
 }

@@ -21,7 +21,7 @@ cudaError_t TOPK_INST_FN(const SelectParams& p, int grid, cudaStream_t st) {
     constexpr bool MIN = TOPK_INST_MIN, FILTER = TOPK_INST_FILTER;
     constexpr int Q = TOPK_INST_Q;
     static std::atomic<bool> attr_set{false};  // idempotent
-    const size_t smem = select_smem_bytes<Key>();
+    const size_t smem = select_smem_bytes<Key, Q>();
     if (!attr_set.load(std::memory_order_relaxed)) {
         cudaError_t e = cudaFuncSetAttribute(select_kernel<Key, MIN, FILTER, Q>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
