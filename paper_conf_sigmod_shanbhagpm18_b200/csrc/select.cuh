@@ -58,6 +58,7 @@ constexpr int kNC = 480;                                    // consumer threads 
 constexpr int kNT = kNC + 32;                               // + one producer warp
 constexpr int kTileBytes = kNC * 16 * TOPK_VEC_PER_THREAD;  // 30 KB per TMA stage
 constexpr int kStagesMax = TOPK_STAGES;
+constexpr int kSmemBudget = 227 * 1024 - 3 * 1024;  // dynamic smem (227 KB opt-in - static)
 constexpr int kCap = 4096;            // survivor buffer entries (incl. the running run)
 constexpr int kPubRows = 11;          // published 2^j-th best for j <= 10 (k up to 2048)
 constexpr int kGMax = 160;            // CTAs (>= SM count)
@@ -101,11 +102,16 @@ struct QCfg {
     // ring: a query stage is TK rows of every column (<= one plain stage), so the ring
     // budget of the plain form holds more of them (up to kStagesMax)
     static constexpr int kSlotBytes = Q == 0 ? kTileBytes : (kTileKeys * kRowBytes + 127) / 128 * 128;
+    // query forms: as many stages as fit next to the buffer, the sample scratch and the
+    // code network (bytes in flight: a KKKV stage is only 23 KB), up to kStagesMax
+    using E_ = typename KeyTraits<Key>::E;
+    static constexpr int kOther = kCap * SBuf<E_>::kBytes + kScratch * 8 +
+                                  (kCap / 512) * 512 * static_cast<int>(sizeof(typename CodeOf<E_>::C)) +
+                                  2 * kStagesMax * 8;
+    static constexpr int kFit = (kSmemBudget - kOther) / kSlotBytes;
     static constexpr int kStages =
-        Q == 0 ? Cfg<Key>::kStages
-               : (Cfg<Key>::kStages * kTileBytes / kSlotBytes < kStagesMax
-                      ? Cfg<Key>::kStages * kTileBytes / kSlotBytes
-                      : kStagesMax);
+        Q == 0 ? Cfg<Key>::kStages : (kFit < kStagesMax ? kFit : kStagesMax);
+    static_assert(kStages >= 2, "ring");
     static_assert(kTileKeys % 4 == 0, "TMA sizes are multiples of 16 bytes");
 };
 
