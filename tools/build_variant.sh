@@ -1,6 +1,14 @@
 #!/bin/bash
 # build_variant.sh NAME "-DMACRO=.. ..."  -> paper_conf_sigmod_shanbhagpm18_b200/variants/libtopk_NAME.so
+# (load it with TOPK_LIB=<path>; dev tool for A/B runs of compile-time knobs)
 set -e
 cd "$(dirname "$0")/.."
-mkdir -p paper_conf_sigmod_shanbhagpm18_b200/variants
-/usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 --shared -Xcompiler -fPIC -diag-suppress 177 $2 -I include -o paper_conf_sigmod_shanbhagpm18_b200/variants/libtopk_$1.so paper_conf_sigmod_shanbhagpm18_b200/csrc/topk_api.cu
+python - "$1" "$2" <<'PY'
+import os, sys
+from paper_conf_sigmod_shanbhagpm18_b200 import _build
+name, flags = sys.argv[1], sys.argv[2].split()
+vdir = os.path.join(_build.PKG, "variants")
+os.makedirs(vdir, exist_ok=True)
+print(_build.build(force=True, extra_flags=flags, lib=os.path.join(vdir, f"libtopk_{name}.so"),
+                   objdir=os.path.join(vdir, f"build_{name}")))
+PY
