@@ -17,19 +17,15 @@ cudaError_t radix_seq(const RadixParams& p, cudaStream_t st) {
                                              cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              static_cast<int>(kMergeSmem));
         if (e != cudaSuccess) return e;
-        for (auto f : {radix_hist<Key, MIN, true>, radix_hist<Key, MIN, false>}) {
-            e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                     static_cast<int>(kHistSmem));
-            if (e != cudaSuccess) return e;
-        }
+
         attr = true;
     }
     const int G = static_cast<int>(p.G);
-    radix_hist<Key, MIN, true><<<G, kHistNT, kHistSmem, st>>>(p);
+    radix_hist<Key, MIN, true><<<G, kHistNT, 0, st>>>(p);
     radix_choose<C, true><<<1, kRadixBins, 0, st>>>(p);
     radix_scatter<Key, MIN><<<G, kRadixNT, 0, st>>>(p);
     for (int d = 1; d < static_cast<int>(sizeof(C)); ++d) {  // the remaining digits
-        radix_hist<Key, MIN, false><<<G, kHistNT, kHistSmem, st>>>(p);
+        radix_hist<Key, MIN, false><<<G, kHistNT, 0, st>>>(p);
         radix_choose<C, false><<<1, kRadixBins, 0, st>>>(p);
         radix_scatter<Key, MIN><<<G, kRadixNT, 0, st>>>(p);
     }

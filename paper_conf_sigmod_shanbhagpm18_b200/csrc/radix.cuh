@@ -209,24 +209,20 @@ __device__ __forceinline__ void warp_append(RadixEntry<C>* list, uint32_t* cnt, 
 
 // Digit pass: per-CTA histogram of digit `shift` over the candidates -- the input
 // filtered by the known prefix (pass 1, or while no bucket was written), else the
-// bucket.  Counts only; the choice is made by radix_choose.  Counters are private per
-// lane (u16 [warp][bin][lane]: bank = lane, no atomics, no conflicts) -- U(0,1) floats
-// put half the keys on one first digit, where shared atomics would serialise.  A lane
-// counts at most slice / kHistNT < 2^16 keys (radix_plan).
-constexpr int kHistNT = 128;
-constexpr size_t kHistSmem = size_t(kHistNT / 32) * kRadixBins * 32 * sizeof(uint16_t);  // 64 KB
+// bucket.  Counts only; the choice is made by radix_choose.  One 256-bin histogram
+// per warp in shared memory, fire-and-forget shared atomics (no result is waited for,
+// so a thread's 16 increments pipeline; same-bin lanes serialise in the atomic unit --
+// U(0,1) floats put half the keys on one first digit), warps summed at the end.
+constexpr int kHistNT = 256;
+constexpr size_t kHistSmem = size_t(kHistNT / 32) * kRadixBins * sizeof(uint32_t);  // 8 KB
 template <class Key, bool MIN, bool FIRST>
 __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
     using C = typename CodeOf<typename KeyTraits<Key>::E>::C;
-    extern __shared__ __align__(16) uint16_t hl[];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    __shared__ uint32_t hw[kHistNT / 32][kRadixBins];
+    const int warp = threadIdx.x >> 5;
     const RadixWs<C> w = radix_ws<C>(p.ws, p.G, p.k);
-    {
-        uint4* z = reinterpret_cast<uint4*>(hl);
-        for (int i = threadIdx.x; i < static_cast<int>(kHistSmem / 16); i += kHistNT)
-            z[i] = make_uint4(0u, 0u, 0u, 0u);
-    }
-    uint16_t* mine = hl + static_cast<size_t>(warp) * kRadixBins * 32 + lane;
+    for (int i = threadIdx.x; i < (kHistNT / 32) * kRadixBins; i += kHistNT) (&hw[0][0])[i] = 0u;
+    uint32_t* mine = hw[warp];
     const C prefix = FIRST ? C(0) : w.st->prefix;
     const uint32_t shift = FIRST ? sizeof(C) * 8 - 8 : w.st->shift;
     const bool from_bucket = !FIRST && w.st->bucket_ok;
@@ -235,34 +231,27 @@ __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
         const uint32_t nb = w.st->nbucket;
         for (uint32_t i = blockIdx.x * kHistNT + threadIdx.x; i < nb; i += gridDim.x * kHistNT) {
             const C c = w.bucket[i].code;
-            if (has_prefix(c, prefix, shift)) mine[digit_of(c, shift) * 32] += 1;
+            if (has_prefix(c, prefix, shift)) atomicAdd(&mine[digit_of(c, shift)], 1u);
         }
     } else {
         const Key* keys = static_cast<const Key*>(p.keys);
         const uint64_t lo = blockIdx.x * p.slice, hi = min(p.n, lo + p.slice);
         constexpr int kT = kHistNT * kRadixPerThread;
-        // two tiles per iteration, both loaded before either is counted (bytes in flight)
-        for (uint64_t t0 = lo; t0 < hi; t0 += 2 * kT) {
-            C c[kRadixPerThread], c2[kRadixPerThread];
-            const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread, r1 = r0 + kT;
+        for (uint64_t t0 = lo; t0 < hi; t0 += kT) {
+            C c[kRadixPerThread];
+            const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
             load_codes<Key, MIN>(keys, hi, r0, c);
-            load_codes<Key, MIN>(keys, hi, r1, c2);
 #pragma unroll
             for (int q = 0; q < kRadixPerThread; ++q)
-                if (r0 + q < hi && has_prefix(c[q], prefix, shift)) mine[digit_of(c[q], shift) * 32] += 1;
-#pragma unroll
-            for (int q = 0; q < kRadixPerThread; ++q)
-                if (r1 + q < hi && has_prefix(c2[q], prefix, shift)) mine[digit_of(c2[q], shift) * 32] += 1;
+                if (r0 + q < hi && has_prefix(c[q], prefix, shift))
+                    atomicAdd(&mine[digit_of(c[q], shift)], 1u);
         }
     }
     __syncthreads();
     for (int b = threadIdx.x; b < kRadixBins; b += kHistNT) {
         uint32_t s = 0;
-        for (int wv = 0; wv < kHistNT / 32; ++wv) {
-            const uint16_t* row = hl + (static_cast<size_t>(wv) * kRadixBins + b) * 32;
-#pragma unroll 8
-            for (int l = 0; l < 32; ++l) s += row[(l + b) & 31];  // rotate: spread banks
-        }
+#pragma unroll
+        for (int wv = 0; wv < kHistNT / 32; ++wv) s += hw[wv][b];
         w.hist[static_cast<size_t>(blockIdx.x) * kRadixBins + b] = s;
     }
 }

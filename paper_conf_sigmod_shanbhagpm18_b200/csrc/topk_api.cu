@@ -404,11 +404,8 @@ struct RadixPlan {
 };
 static RadixPlan radix_plan(uint64_t n, int sms) {
     RadixPlan r;
-    // 3 histogram CTAs (128 threads, 64 KB of lane-private u16 counters) per SM, and
-    // enough slices that one lane counts < 2^16 keys of its slice
-    uint64_t g = 3ull * static_cast<uint64_t>(sms);
-    const uint64_t gmin = (n + 60000ull * topk::kHistNT - 1) / (60000ull * topk::kHistNT);
-    if (g < gmin) g = gmin;
+    // 4 CTAs of 256 threads per SM, one contiguous slice each
+    const uint64_t g = 4ull * static_cast<uint64_t>(sms);
     uint64_t slice = (n + g - 1) / g;
     slice = (slice + topk::kRadixTile - 1) / topk::kRadixTile * topk::kRadixTile;
     r.slice = slice;
