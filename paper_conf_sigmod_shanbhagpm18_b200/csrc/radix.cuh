@@ -75,12 +75,12 @@ struct RadixParams {
     int64_t* out_idx;
 };
 
-// Workspace layout: [state | hist G x 256 | gt k | eq kRadixEqCap | eqc G x k |
+// Workspace layout: [state | hist 256 (+ spare) | gt k | eq kRadixEqCap | eqc G x k |
 // eqn G | bucket cap].
 template <class C>
 struct RadixWs {
     RadixState<C>* st;
-    uint32_t* hist;
+    uint32_t* hist;  // [256] digit totals of the current pass
     RadixEntry<C>* gt;
     RadixEntry<C>* eq;
     RadixEntry<C>* eqc;
@@ -252,7 +252,7 @@ __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
         uint32_t s = 0;
 #pragma unroll
         for (int wv = 0; wv < kHistNT / 32; ++wv) s += hw[wv][b];
-        w.hist[static_cast<size_t>(blockIdx.x) * kRadixBins + b] = s;
+        if (s) atomicAdd(&w.hist[b], s);  // the pass's total (radix_choose reads and zeroes it)
     }
 }
 
@@ -267,7 +267,8 @@ __global__ void __launch_bounds__(kRadixBins) radix_choose(const RadixParams p) 
     RadixState<C>* st = w.st;
     const int d = threadIdx.x;
     uint32_t s = 0;
-    for (uint32_t c = 0; c < p.G; ++c) s += w.hist[static_cast<size_t>(c) * kRadixBins + d];
+    s = w.hist[d];
+    w.hist[d] = 0u;  // ready for the next digit pass
     tot[d] = s;
     __syncthreads();
     if (d == 0) {
@@ -340,15 +341,21 @@ __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
         C c[kRadixPerThread];
         const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
         load_codes<Key, MIN>(keys, hi, r0, c);
-        uint32_t nb = 0;
+        uint32_t nb = 0, gtm = 0;
 #pragma unroll
         for (int q = 0; q < kRadixPerThread; ++q) {
             const bool ok = r0 + q < hi;
             const C dg = c[q] >> kTop;  // code above the bucket's bits
             nb += (ok && dg == d1) ? 1u : 0u;
-            // entries above the bucket: fewer than k in all (rare: warp-aggregated)
-            warp_append(w.gt, &w.st->ngt, p.k, ok && dg > d1,
-                        RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)}, nullptr);
+            gtm |= static_cast<uint32_t>(ok && dg > d1) << q;
+        }
+        // entries above the bucket: fewer than k in all (rare: one vote per tile, then
+        // warp-aggregated appends)
+        if (__any_sync(0xFFFFFFFFu, gtm != 0u)) {
+#pragma unroll
+            for (int q = 0; q < kRadixPerThread; ++q)
+                warp_append(w.gt, &w.st->ngt, p.k, (gtm >> q) & 1u,
+                            RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)}, nullptr);
         }
         uint32_t tile_nb;
         const uint32_t off = block_excl_scan(nb, s_w, &tile_nb);
