@@ -438,7 +438,7 @@ static __device__ __constant__ int c_trace_on;  // set by topk_debug_trace (cons
 // bit 1 -- no boot-time wait for peers; bit 2 -- no early second flush; bit 3 -- no
 // small-buffer exact network (wnet_small); bits 4-5 -- rank-bound rows (0 = 3);
 // bits 6-7 -- second-flush limit 512 * (1 + v) (0 = TOPK_LIMIT2); bits 8-9 -- boot
-// buffer kCap >> v (0 = by K: 512 for K >= 256, else 4096).
+// buffer kCap >> v, bits 8-10 (0 = by K: 512 for K >= 256, else 4096).
 static __device__ __constant__ int c_dbg;
 __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
@@ -1132,7 +1132,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // large K -- whose flush costs more -- boots on a small sample (measured with the
         // c_dbg knob, 2^29 uniform f32: K >= 256 best with 512 entries -- k = 256 379 ->
         // 363 us, k = 1024 406 -> 396 us; K <= 128 best with the whole buffer)
-        st.limit = (c_dbg >> 8) & 3 ? kCap >> ((c_dbg >> 8) & 3)
+        st.limit = (c_dbg >> 8) & 7 ? kCap >> ((c_dbg >> 8) & 7)
                    : K >= 256 ? kCap / 8 : kCap;
         st.ties = 0;
         st.tau_w = 0ull;
