@@ -640,8 +640,10 @@ __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
     // size: every CTA meets the ties at about the same time, and a 4096-entry exact
     // flush idles the HBM for ~20 us (measured, k = 256: few-distinct 430 -> 392 us,
     // bucket killer 432 -> ~395 us).  c_dbg bits 11-12 override the shift (default 3).
+    // Progress: the bag must take a warp's largest append (32 lanes x 16 keys = 512)
+    // on top of the K entries an exact flush keeps.
     const int tl = (c_dbg >> 11) & 3 ? (c_dbg >> 11) & 3 : 3;
-    if (ties) return max(2 * K, kCap >> tl);
+    if (ties) return max(max(2 * K, K + 512), kCap >> tl);
     return (nflush == 1 && Lp >= 0 && !(c_dbg & 4)) ? max(l2, 2 * K) : kCap;
 }
 
