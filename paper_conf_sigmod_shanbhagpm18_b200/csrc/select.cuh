@@ -634,16 +634,9 @@ __device__ int compact_bag(const SBuf<E>& buf, int cnt, E tau, int* s_w) {
 // one buffer per CTA only) and the rank bound tightens early.  A stream flush always
 // leaves at most half of the next limit (progress: a warp appends <= 512 at a time).
 __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
+    (void)ties;
     // (K = 256: 2K = 512 measured 6 us faster than 1024; other K: no difference)
     const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3)) : K == 256 ? 512 : TOPK_LIMIT2;
-    // tie-heavy bags (the code path failed: equal keys) are flushed exactly at a small
-    // size: every CTA meets the ties at about the same time, and a 4096-entry exact
-    // flush idles the HBM for ~20 us (measured, k = 256: few-distinct 430 -> 392 us,
-    // bucket killer 432 -> ~395 us).  c_dbg bits 11-12 override the shift (default 3).
-    // Progress: the bag must take a warp's largest append (32 lanes x 16 keys = 512)
-    // on top of the K entries an exact flush keeps.
-    const int tl = (c_dbg >> 11) & 3 ? (c_dbg >> 11) & 3 : 3;
-    if (ties) return max(max(2 * K, K + 512), kCap >> tl);
     return (nflush == 1 && Lp >= 0 && !(c_dbg & 4)) ? max(l2, 2 * K) : kCap;
 }
 
