@@ -634,9 +634,13 @@ __device__ int compact_bag(const SBuf<E>& buf, int cnt, E tau, int* s_w) {
 // one buffer per CTA only) and the rank bound tightens early.  A stream flush always
 // leaves at most half of the next limit (progress: a warp appends <= 512 at a time).
 __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
-    (void)ties;
     // (K = 256: 2K = 512 measured 6 us faster than 1024; other K: no difference)
     const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3)) : K == 256 ? 512 : TOPK_LIMIT2;
+    // Tie-heavy bags (the code path failed on equal keys) flush exactly at a small size:
+    // every CTA meets the ties at about the same time and a 4096-entry exact flush idles
+    // the HBM for ~20 us.  Progress: room for a warp's largest append (32 lanes x 16
+    // keys = 512) on top of the K entries an exact flush keeps.
+    if (ties) return max(max(2 * K, K + 512), kCap >> 3);
     return (nflush == 1 && Lp >= 0 && !(c_dbg & 4)) ? max(l2, 2 * K) : kCap;
 }
 
