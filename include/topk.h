@@ -31,8 +31,9 @@
  *     memory, never frees, and retains no pointer after the call returns.  Buffers must
  *     stay valid until the stream reaches the enqueued work.
  *   - Workspace: `ws` of at least topk_workspace_bytes(...) bytes, 256-byte aligned,
- *     zero-filled before its FIRST use (topk_workspace_init); every call leaves it
- *     zero-filled again.  One workspace must not be used by two calls concurrently;
+ *     zero-filled before its FIRST use (topk_workspace_init); every call leaves its
+ *     control words zeroed again (the candidate area is scratch), so it needs no
+ *     re-initialisation between calls.  One workspace must not be used by two calls concurrently;
  *     calls with distinct workspaces are re-entrant.
  *   - Errors: argument errors are returned synchronously and nothing is enqueued;
  *     launch failures return TOPK_ERR_CUDA; asynchronous faults surface at the caller's
@@ -223,7 +224,8 @@ topk_status_t topk_select_host(topk_dtype_t dtype, const void* h_keys, uint64_t 
  * back to back: cand_keys[runs*run_len] (key type), cand_idx[runs*run_len] int64
  * global row ids (the tie-break), cand_payload optional.  Entries may be in any order;
  * duplicated (key, idx) entries are not allowed.  1 <= k <= min(runs*run_len, 2048),
- * runs*run_len <= 65536.  Single-CTA merge + rebuild network; ws as topk_merge_ws_bytes. */
+ * runs*run_len <= 65536.  Single-CTA local sort + merge + rebuild network (in chunks of
+ * 4096 entries next to the running top-k); ws as topk_merge_workspace_bytes (unused). */
 size_t topk_merge_workspace_bytes(topk_dtype_t dtype, uint32_t runs, uint32_t run_len,
                                   uint32_t k);
 topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_t* cand_idx,
@@ -231,6 +233,18 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
                          uint32_t k, topk_order_t order, void* out_keys,
                          uint32_t* out_payload, int64_t* out_idx, void* ws,
                          size_t ws_bytes, void* stream);
+
+/* topk_merge for candidates whose every run is sorted best first -- the order every
+ * topk_select / topk_* result has (the multi-GPU all-gather, chunked inputs): the kernel
+ * skips the local sort and runs log2(runs) rounds of the paper's merge + rebuild over
+ * the runs (run 2i as is, run 2i+1 reversed: each pair is one bitonic sequence, P:150;
+ * Alg. 4).  Same arguments and result as topk_merge; a run's entries past position
+ * next_pow2(k) are never read.  Passing unsorted runs gives an unspecified result. */
+topk_status_t topk_merge_sorted(topk_dtype_t dtype, const void* cand_keys,
+                                const int64_t* cand_idx, const uint32_t* cand_payload,
+                                uint32_t runs, uint32_t run_len, uint32_t k, topk_order_t order,
+                                void* out_keys, uint32_t* out_payload, int64_t* out_idx,
+                                void* ws, size_t ws_bytes, void* stream);
 
 /* ---- Multi-GPU: the partitioned top-k (§1 "per-partition top-k ... global top-k
  * from the m per-partition heaps"; App. C "combined in a final global step") ----

@@ -38,6 +38,28 @@ def _ptr(t):
     return ctypes.c_void_p(t.data_ptr()) if t is not None else None
 
 
+def _check_col(t, n, dtype, device, what):
+    """A CUDA column the kernels read: dtype, length, device and layout are checked here,
+    so a wrong tensor raises instead of turning into an out-of-bounds device access."""
+    if t is None:
+        return None
+    if not t.is_cuda or t.device != device:
+        raise ValueError(f"{what}: must be a CUDA tensor on {device}")
+    if t.dtype != dtype or t.dim() != 1 or t.shape[0] != n:
+        raise ValueError(f"{what}: expected a 1-D {dtype} tensor of length {n}")
+    return t.contiguous()
+
+
+def _check_out(t, k, dtype, device, what):
+    if t is None:
+        return None
+    if not t.is_cuda or t.device != device or t.dtype != dtype or t.numel() < k \
+            or not t.is_contiguous():
+        raise ValueError(f"{what}: expected a contiguous CUDA {dtype} tensor of >= {k} "
+                         f"elements on {device}")
+    return t
+
+
 def workspace_bytes(dtype: torch.dtype, n: int, k: int) -> int:
     return int(_lib.load().topk_workspace_bytes(_DT[dtype], n, k))
 
@@ -80,25 +102,31 @@ def topk(x: torch.Tensor, k: int, largest: bool = True, payload: torch.Tensor | 
     dt = _dtype_code(x)
     n = x.shape[0]
     x = x if x.is_contiguous() else x.contiguous()
+    if mode not in ("filter", "pure"):
+        raise ValueError(f"mode must be 'filter' or 'pure', not {mode!r}")
+    dev = x.device
+    payload = _check_col(payload, n, torch.uint32, dev, "payload")
     if out is None:
-        vals = torch.empty(k, dtype=x.dtype, device=x.device)
-        idx = torch.empty(k, dtype=torch.int64, device=x.device)
-        pay = torch.empty(k, dtype=torch.uint32, device=x.device) if payload is not None else None
+        vals = torch.empty(k, dtype=x.dtype, device=dev)
+        idx = torch.empty(k, dtype=torch.int64, device=dev)
+        pay = torch.empty(k, dtype=torch.uint32, device=dev) if payload is not None else None
     else:
         vals, idx, pay = out
-    if payload is not None:
-        if payload.dtype != torch.uint32 or payload.shape[0] != n or not payload.is_cuda:
-            raise ValueError("payload must be a CUDA uint32 tensor of the same length")
-        payload = payload.contiguous()
-    need = int(lib.topk_workspace_bytes(dt, n, k))
-    if need == 0:
-        raise _lib.TopkError(f"invalid arguments for topk (n={n}, k={k})")
-    ws = workspace if workspace is not None else _workspace(x.device, need)
-    st = lib.topk_select(dt, _ptr(x), _ptr(payload), n, base, k,
-                         _lib.LARGEST if largest else _lib.SMALLEST,
-                         _lib.MODE_FILTER if mode == "filter" else _lib.MODE_PURE,
-                         _ptr(vals), _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
-                         _stream_ptr(x.device))
+        vals = _check_out(vals, k, x.dtype, dev, "out values")
+        idx = _check_out(idx, k, torch.int64, dev, "out indices")
+        pay = _check_out(pay, k, torch.uint32, dev, "out payload")
+        if pay is not None and payload is None:
+            raise ValueError("out payload given without an input payload")
+    with torch.cuda.device(dev):
+        need = int(lib.topk_workspace_bytes(dt, n, k))
+        if need == 0:
+            raise _lib.TopkError(f"invalid arguments for topk (n={n}, k={k})")
+        ws = workspace if workspace is not None else _workspace(dev, need)
+        st = lib.topk_select(dt, _ptr(x), _ptr(payload), n, base, k,
+                             _lib.LARGEST if largest else _lib.SMALLEST,
+                             _lib.MODE_FILTER if mode == "filter" else _lib.MODE_PURE,
+                             _ptr(vals), _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
+                             _stream_ptr(dev))
     _lib.check(st, "topk_select")
     return (vals, idx) if payload is None else (vals, idx, pay)
 
@@ -137,20 +165,22 @@ def query(keys: torch.Tensor, k: int, largest: bool = True, rank_b: torch.Tensor
             raise ValueError("rank_b: contiguous CUDA float32 of the same length")
         cols.append(rank_b)
     if payload is not None:
+        payload = _check_col(payload, n, torch.uint32, keys.device, "payload")
         cols.append(payload)
-    if any(not c.is_contiguous() for c in cols):
-        raise ValueError("columns must be contiguous")
+    if any(not c.is_contiguous() or c.device != keys.device for c in cols):
+        raise ValueError("columns must be contiguous and on the keys' device")
     vals = torch.empty(k, dtype=keys.dtype, device=keys.device)
     idx = torch.empty(k, dtype=torch.int64, device=keys.device)
     pay = torch.empty(k, dtype=torch.uint32, device=keys.device) if payload is not None else None
-    need = int(lib.topk_workspace_bytes(dt, n, k))
-    if need == 0:
-        raise _lib.TopkError(f"invalid arguments for query (n={n}, k={k})")
-    ws = workspace if workspace is not None else _workspace(keys.device, need)
-    st = lib.topk_query(dt, _ptr(keys), _ptr(rank_b), float(rank_w),
-                        ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k,
-                        _lib.LARGEST if largest else _lib.SMALLEST, _ptr(vals), _ptr(pay),
-                        _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(keys.device))
+    with torch.cuda.device(keys.device):
+        need = int(lib.topk_workspace_bytes(dt, n, k))
+        if need == 0:
+            raise _lib.TopkError(f"invalid arguments for query (n={n}, k={k})")
+        ws = workspace if workspace is not None else _workspace(keys.device, need)
+        st = lib.topk_query(dt, _ptr(keys), _ptr(rank_b), float(rank_w),
+                            ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k,
+                            _lib.LARGEST if largest else _lib.SMALLEST, _ptr(vals), _ptr(pay),
+                            _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(keys.device))
     _lib.check(st, "topk_query")
     return (vals, idx) if payload is None else (vals, idx, pay)
 
@@ -185,15 +215,19 @@ def topk_kk(k1: torch.Tensor, k2: torch.Tensor, k: int, largest1: bool = True,
     v2 = torch.empty(k, dtype=torch.float32, device=dev)
     idx = torch.empty(k, dtype=torch.int64, device=dev)
     pay = torch.empty(k, dtype=torch.uint32, device=dev) if payload is not None else None
-    need = int(lib.topk_workspace_bytes(_lib.F64, n, k))
-    if need == 0:
-        raise _lib.TopkError(f"invalid arguments for topk_kk (n={n}, k={k})")
-    ws = workspace if workspace is not None else _workspace(dev, need)
-    st = lib.topk_kk(_ptr(k1.contiguous()), _ptr(k2.contiguous()),
-                     ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k,
-                     _lib.LARGEST if largest1 else _lib.SMALLEST,
-                     _lib.LARGEST if largest2 else _lib.SMALLEST, _ptr(v1), _ptr(v2), _ptr(pay),
-                     _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(dev))
+    payload = _check_col(payload, n, torch.uint32, dev, "payload")
+    if k2.device != dev or (pred is not None and pred[1].device != dev):
+        raise ValueError("topk_kk: every column on the same device")
+    with torch.cuda.device(dev):
+        need = int(lib.topk_workspace_bytes(_lib.F64, n, k))
+        if need == 0:
+            raise _lib.TopkError(f"invalid arguments for topk_kk (n={n}, k={k})")
+        ws = workspace if workspace is not None else _workspace(dev, need)
+        st = lib.topk_kk(_ptr(k1.contiguous()), _ptr(k2.contiguous()),
+                         ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k,
+                         _lib.LARGEST if largest1 else _lib.SMALLEST,
+                         _lib.LARGEST if largest2 else _lib.SMALLEST, _ptr(v1), _ptr(v2),
+                         _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(dev))
     _lib.check(st, "topk_kk")
     return (v1, v2, idx) if payload is None else (v1, v2, idx, pay)
 
@@ -214,15 +248,19 @@ def topk_kkk(k1: torch.Tensor, k2: torch.Tensor, k3: torch.Tensor, k: int,
     outs = [torch.empty(k, dtype=torch.float32, device=dev) for _ in range(3)]
     idx = torch.empty(k, dtype=torch.int64, device=dev)
     pay = torch.empty(k, dtype=torch.uint32, device=dev) if payload is not None else None
-    need = int(lib.topk_workspace_bytes(_lib.F64, n, k))
-    if need == 0:
-        raise _lib.TopkError(f"invalid arguments for topk_kkk (n={n}, k={k})")
-    ws = workspace if workspace is not None else _workspace(dev, need)
+    payload = _check_col(payload, n, torch.uint32, dev, "payload")
+    if any(c.device != dev for c in cols) or (pred is not None and pred[1].device != dev):
+        raise ValueError("topk_kkk: every column on the same device")
     o = [_lib.LARGEST if l else _lib.SMALLEST for l in largest]
-    st = lib.topk_kkk(*[_ptr(c.contiguous()) for c in cols],
-                      ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k, *o,
-                      *[_ptr(t) for t in outs], _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
-                      _stream_ptr(dev))
+    with torch.cuda.device(dev):
+        need = int(lib.topk_workspace_bytes(_lib.F64, n, k))
+        if need == 0:
+            raise _lib.TopkError(f"invalid arguments for topk_kkk (n={n}, k={k})")
+        ws = workspace if workspace is not None else _workspace(dev, need)
+        st = lib.topk_kkk(*[_ptr(c.contiguous()) for c in cols],
+                          ctypes.byref(pr) if pr is not None else None, _ptr(payload), n, k, *o,
+                          *[_ptr(t) for t in outs], _ptr(pay), _ptr(idx), ws.ptr(), ws.nbytes,
+                          _stream_ptr(dev))
     _lib.check(st, "topk_kkk")
     return (*outs, idx) if payload is None else (*outs, idx, pay)
 
@@ -236,18 +274,24 @@ def topk_radix(x: torch.Tensor, k: int, largest: bool = True, out=None):
     dt = _dtype_code(x)
     n = x.shape[0]
     x = x.contiguous()
-    need = int(lib.topk_radix_workspace_bytes(dt, n, k))
-    if need == 0:
-        raise _lib.TopkError(f"invalid arguments for topk_radix (n={n}, k={k})")
-    key = ("radix", x.device.index, torch.cuda.current_stream(x.device).cuda_stream)
-    ws = _ws_cache.get(key)
-    if ws is None or ws.nbytes < need:
-        ws = Workspace(need, x.device)
-        _ws_cache[key] = ws
-    vals, idx = out if out is not None else (torch.empty(k, dtype=x.dtype, device=x.device),
-                                             torch.empty(k, dtype=torch.int64, device=x.device))
-    st = lib.topk_radix(dt, _ptr(x), n, k, _lib.LARGEST if largest else _lib.SMALLEST,
-                        _ptr(vals), _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(x.device))
+    dev = x.device
+    if out is not None:
+        vals = _check_out(out[0], k, x.dtype, dev, "out values")
+        idx = _check_out(out[1], k, torch.int64, dev, "out indices")
+    else:
+        vals = torch.empty(k, dtype=x.dtype, device=dev)
+        idx = torch.empty(k, dtype=torch.int64, device=dev)
+    with torch.cuda.device(dev):
+        need = int(lib.topk_radix_workspace_bytes(dt, n, k))
+        if need == 0:
+            raise _lib.TopkError(f"invalid arguments for topk_radix (n={n}, k={k})")
+        key = ("radix", dev.index, torch.cuda.current_stream(dev).cuda_stream)
+        ws = _ws_cache.get(key)
+        if ws is None or ws.nbytes < need:
+            ws = Workspace(need, dev)
+            _ws_cache[key] = ws
+        st = lib.topk_radix(dt, _ptr(x), n, k, _lib.LARGEST if largest else _lib.SMALLEST,
+                            _ptr(vals), _ptr(idx), ws.ptr(), ws.nbytes, _stream_ptr(dev))
     _lib.check(st, "topk_radix")
     return vals, idx
 
@@ -279,34 +323,39 @@ def topk_host(x: torch.Tensor, k: int, largest: bool = True, chunk_keys: int = 1
     else:
         vals, idx = out
     x = x.contiguous()
-    st = lib.topk_select_host(dt, _ptr(x), n, k, _lib.LARGEST if largest else _lib.SMALLEST,
-                              _ptr(vals), _ptr(idx), chunk_keys, ws.ptr(), ws.nbytes,
-                              _stream_ptr(dev))
+    with torch.cuda.device(dev):
+        st = lib.topk_select_host(dt, _ptr(x), n, k, _lib.LARGEST if largest else _lib.SMALLEST,
+                                  _ptr(vals), _ptr(idx), chunk_keys, ws.ptr(), ws.nbytes,
+                                  _stream_ptr(dev))
     _lib.check(st, "topk_select_host")
     return vals, idx
 
 
 def merge(cand_keys: torch.Tensor, cand_idx: torch.Tensor, k: int, largest: bool = True,
-          cand_payload: torch.Tensor | None = None, runs: int = 1):
+          cand_payload: torch.Tensor | None = None, runs: int = 1, sorted_runs: bool = False):
     """Exact top-k of candidate entries (key, global int64 index[, payload]) -- the
-    global step after per-partition top-k (multi-GPU all-gather result)."""
+    global step after per-partition top-k (multi-GPU all-gather result).  With
+    ``sorted_runs`` every one of the ``runs`` equal-length runs must be sorted best first
+    (as :func:`topk` returns them): only the merge + rebuild rounds run."""
+    if not cand_keys.is_cuda or cand_keys.dim() != 1:
+        raise ValueError("merge expects 1-D CUDA candidate tensors (no CPU path)")
     lib = _lib.load()
     dt = _dtype_code(cand_keys)
     total = cand_keys.shape[0]
-    if total % runs:
+    if runs < 1 or total % runs:
         raise ValueError("candidates must be runs * run_len long")
     cand_keys = cand_keys.contiguous()
-    cand_idx = cand_idx.to(torch.int64).contiguous()
     dev = cand_keys.device
+    cand_idx = _check_col(cand_idx, total, torch.int64, dev, "cand_idx")
+    cand_payload = _check_col(cand_payload, total, torch.uint32, dev, "cand_payload")
     vals = torch.empty(k, dtype=cand_keys.dtype, device=dev)
     idx = torch.empty(k, dtype=torch.int64, device=dev)
-    pay = None
-    if cand_payload is not None:
-        cand_payload = cand_payload.contiguous()
-        pay = torch.empty(k, dtype=torch.uint32, device=dev)
-    st = lib.topk_merge(dt, _ptr(cand_keys), _ptr(cand_idx), _ptr(cand_payload), runs,
-                        total // runs, k, _lib.LARGEST if largest else _lib.SMALLEST,
-                        _ptr(vals), _ptr(pay), _ptr(idx), None, 0, _stream_ptr(dev))
+    pay = torch.empty(k, dtype=torch.uint32, device=dev) if cand_payload is not None else None
+    with torch.cuda.device(dev):
+        fn = lib.topk_merge_sorted if sorted_runs else lib.topk_merge
+        st = fn(dt, _ptr(cand_keys), _ptr(cand_idx), _ptr(cand_payload), runs,
+                total // runs, k, _lib.LARGEST if largest else _lib.SMALLEST,
+                _ptr(vals), _ptr(pay), _ptr(idx), None, 0, _stream_ptr(dev))
     _lib.check(st, "topk_merge")
     return (vals, idx) if cand_payload is None else (vals, idx, pay)
 

@@ -21,7 +21,7 @@ MODE_FILTER, MODE_PURE = 0, 1
 # Every symbol include/topk.h declares (tests check the .so exports all of them).
 SYMBOLS = (
     "topk_workspace_bytes", "topk_workspace_init", "topk_select", "topk_f32", "topk_u32",
-    "topk_f64", "topk_u32_kv", "topk_f64_kv", "topk_merge_workspace_bytes", "topk_merge",
+    "topk_f64", "topk_u32_kv", "topk_f64_kv", "topk_merge_workspace_bytes", "topk_merge", "topk_merge_sorted",
     "topk_launch_count", "topk_status_string", "topk_abi_version", "topk_probe_read",
     "topk_host_workspace_bytes", "topk_select_host", "topk_nccl_unique_id", "topk_nccl_comm_init",
     "topk_nccl_comm_destroy", "topk_sharded_workspace_bytes", "topk_select_sharded",
@@ -73,6 +73,8 @@ def load(build_if_missing: bool = True):
     lib.topk_merge_workspace_bytes.restype = sz
     lib.topk_merge.argtypes = [i32, vp, vp, vp, u32, u32, u32, i32, vp, vp, vp, vp, sz, vp]
     lib.topk_merge.restype = i32
+    lib.topk_merge_sorted.argtypes = [i32, vp, vp, vp, u32, u32, u32, i32, vp, vp, vp, vp, sz, vp]
+    lib.topk_merge_sorted.restype = i32
     lib.topk_probe_read.argtypes = [vp, sz, i32, i32, i32, i32, vp, vp]
     lib.topk_probe_read.restype = i32
     lib.topk_host_workspace_bytes.argtypes = [i32, u64, u32, u64]

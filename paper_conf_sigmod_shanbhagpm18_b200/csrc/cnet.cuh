@@ -26,6 +26,7 @@
 // change costs one XOR per code instead of a select per compare-exchange.
 #pragma once
 #include "keys.cuh"
+#include "network.cuh"
 
 namespace topk {
 
@@ -248,6 +249,28 @@ __device__ void cnet_topk_codes(const SBuf<E>& b, int n, int Lp, typename CodeOf
         }
         Sync::sync();
     }
+}
+
+}  // namespace topk
+
+namespace topk {
+
+// Test hook: the code-only network on n caller-supplied codes (one CTA of the consumer
+// shape); writes the top-2^Lp codes best first to out (topk_debug_cnet, used by the
+// order-statistics parity test).
+template <class E, int NW>
+__global__ void __launch_bounds__(NW * 32, 1) cnet_debug_kernel(
+    const typename CodeOf<E>::C* codes, int n, int Lp, typename CodeOf<E>::C* out) {
+    using C = typename CodeOf<E>::C;
+    extern __shared__ __align__(128) unsigned char smem[];
+    SBuf<E> b;
+    b.init(smem, 4096);
+    C* S = reinterpret_cast<C*>(smem + 4096 * 12);
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    for (int i = threadIdx.x; i < n; i += NW * 32) b.st(i, E::make(codes[i], static_cast<uint32_t>(i)));
+    NamedSync<NW * 32>::sync();
+    cnet_topk_codes<E, NW, NamedSync<NW * 32>>(b, n, Lp, S, w, lane);
+    for (int j = threadIdx.x; j < (1 << Lp); j += NW * 32) out[j] = S[j];
 }
 
 }  // namespace topk

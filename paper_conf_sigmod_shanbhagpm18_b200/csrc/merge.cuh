@@ -1,12 +1,25 @@
 // merge.cuh -- the global step of the partitioned top-k: "computing the global top-k
 // from the m per-partition heaps" (§1), "the top-k elements emitted by the
-// individual core are combined in a final global step" (App. C).  Used for the
-// multi-GPU path (§8(e)): G ranks' candidate runs -> one exact top-k, with the same
-// local sort / merge / rebuild network (network.cuh) over entries that carry a 64-bit
-// global index as the tie-break.
+// individual core are combined in a final global step" (App. C).  Used after the
+// multi-GPU all-gather (§8(e)), after the chunks of an input longer than one launch, and
+// after the chunks of a host-resident input.
+//
+// The candidates arrive as G runs.  When each run is already sorted best first (every
+// topk_select result is), the kernel skips the local sort: run 2i is loaded as it is and
+// run 2i+1 reversed, so every pair is one bitonic sequence -- exactly the state the
+// paper's local sort leaves (Alg. 2: runs alternating direction) -- and log2 G rounds of
+// merge (keep the better of paired elements) + rebuild (Alg. 4) leave
+// the top-K best first.  Unsorted candidates (topk_merge's general contract) run the
+// local sort first.  Inputs with more than one buffer of runs are folded in chunks: the
+// running top-K stays in run slot 0 and the next runs fill the other slots.
+//
+// Entries carry the 64-bit global index as the tie-break (R1) and the row of
+// the candidate array for the output gather.  One CTA, entries in registers (R per
+// lane) with warp shuffles / shared-memory exchanges (wnet.cuh wnet_small).
 #pragma once
 #include "keys.cuh"
 #include "network.cuh"
+#include "wnet.cuh"
 
 namespace topk {
 
@@ -22,6 +35,15 @@ __device__ __forceinline__ bool better(EM a, EM b) {
 }
 __device__ __forceinline__ EM esel(bool p, EM a, EM b) {
     return EM{sel64(p, a.c, b.c), sel64(p, a.idx, b.idx), sel32(p, a.row, b.row)};
+}
+template <>
+__device__ __forceinline__ EM shfl_xor_e<EM>(const EM& e, int m) {
+    const uint32_t c0 = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.c), m);
+    const uint32_t c1 = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.c >> 32), m);
+    const uint32_t i0 = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.idx), m);
+    const uint32_t i1 = __shfl_xor_sync(0xFFFFFFFFu, static_cast<uint32_t>(e.idx >> 32), m);
+    const uint32_t r = __shfl_xor_sync(0xFFFFFFFFu, e.row, m);
+    return EM{(static_cast<uint64_t>(c1) << 32) | c0, (static_cast<uint64_t>(i1) << 32) | i0, r};
 }
 template <>
 struct SBuf<EM> {
@@ -40,12 +62,24 @@ struct SBuf<EM> {
         idx[i] = e.idx;
         row[i] = e.row;
     }
+    __device__ __forceinline__ void ld2(int i, EM& a, EM& b) const {  // i even
+        const ulonglong2 q = *reinterpret_cast<const ulonglong2*>(c + i);
+        const ulonglong2 x = *reinterpret_cast<const ulonglong2*>(idx + i);
+        const uint2 r = *reinterpret_cast<const uint2*>(row + i);
+        a = EM{q.x, x.x, r.x};
+        b = EM{q.y, x.y, r.y};
+    }
+    __device__ __forceinline__ void st2(int i, EM a, EM b) const {
+        *reinterpret_cast<ulonglong2*>(c + i) = make_ulonglong2(a.c, b.c);
+        *reinterpret_cast<ulonglong2*>(idx + i) = make_ulonglong2(a.idx, b.idx);
+        *reinterpret_cast<uint2*>(row + i) = make_uint2(a.row, b.row);
+    }
 };
 
-constexpr int kMergeNT = 512;
-constexpr int kMergeCap = 8192;
-constexpr int kMergeChunk = 4096;
-constexpr size_t kMergeSmem = static_cast<size_t>(kMergeCap) * SBuf<EM>::kBytes;
+constexpr int kMergeNT = 512;                     // 16 warps
+constexpr int kMergeP = 4096;                     // entries per network buffer
+constexpr int kMergeCap = 2 * kMergeP;            // + the exchange region of wnet_small
+constexpr size_t kMergeSmem = static_cast<size_t>(kMergeCap) * SBuf<EM>::kBytes;  // 160 KB
 
 struct MergeParams {
     const void* cand_keys;
@@ -54,72 +88,89 @@ struct MergeParams {
     void* out_keys;
     uint32_t* out_payload;
     int64_t* out_idx;
-    uint32_t total;  // runs * run_len
+    uint32_t total;    // candidate entries (runs of run_len, the last one may be shorter)
+    uint32_t run_len;  // entries per run
+    uint32_t sorted;   // 1: every run is sorted best first (topk_select's output order)
     uint32_t k, K;
 };
+
+// The network over b[0 .. P) (wnet_small: R entries per lane, W = P / (32 R) warps).
+template <class Sync>
+__device__ __forceinline__ void merge_net(const SBuf<EM>& b, int P, int L, bool presorted, int w,
+                                          int lane) {
+    if (P <= 1024)
+        wnet_small<EM, 2, kMergeNT / 32, Sync>(b, P, L, w, lane, presorted);
+    else if (P <= 2048)
+        wnet_small<EM, 4, kMergeNT / 32, Sync>(b, P, L, w, lane, presorted);
+    else
+        wnet_small<EM, 8, kMergeNT / 32, Sync>(b, P, L, w, lane, presorted);
+}
 
 template <class Key, bool MIN>
 __global__ void __launch_bounds__(kMergeNT, 1) merge_kernel(const MergeParams p) {
     using KT = KeyTraits<Key>;
     extern __shared__ __align__(128) unsigned char smem[];
-    __shared__ int s_cnt;
-    SBuf<EM> buf;
-    buf.init(smem, kMergeCap);
-    const int tid = threadIdx.x, lane = tid & 31;
+    SBuf<EM> b;
+    b.init(smem, kMergeCap);
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
     const int K = static_cast<int>(p.K), k = static_cast<int>(p.k);
-    const int flush_at = kMergeCap - K - kMergeChunk;
+    const int L = __ffs(K) - 1;
     const Key* ck = static_cast<const Key*>(p.cand_keys);
-    for (int i = tid; i < K; i += kMergeNT) buf.st(i, EM::sentinel());
-    if (tid == 0) s_cnt = 0;
-    __syncthreads();
-
-    auto do_flush = [&]() {
-        const int cnt = s_cnt;
-        int P = K + cnt <= 1 ? 1 : 1 << (32 - __clz(K + cnt - 1));
-        if (P < 2 * K) P = 2 * K;
-        for (int i = K + cnt + tid; i < P; i += kMergeNT) buf.st(i, EM::sentinel());
-        __syncthreads();
-        bitonic_topk_smem<EM, kMergeNT, CtaSync>(buf, P, K);
-        if (tid == 0) s_cnt = 0;
-        __syncthreads();
+    auto entry = [&](uint32_t q) -> EM {
+        return EM{static_cast<uint64_t>(KT::template code<MIN>(ck[q])),
+                  static_cast<uint64_t>(p.cand_idx[q]), q};
     };
-
-    constexpr int CI = kMergeChunk / kMergeNT;
-    for (uint32_t q0 = 0; q0 < p.total; q0 += kMergeChunk) {
-        // Append every candidate of this chunk (warp-aggregated prefix sum).
-        int cnt = 0;
-        EM ents[CI];
-#pragma unroll
-        for (int r = 0; r < CI; ++r) {
-            const uint32_t q = q0 + tid + r * kMergeNT;
-            ents[r] = EM::sentinel();
-            if (q < p.total) {
-                ents[r] = EM{static_cast<uint64_t>(KT::template code<MIN>(ck[q])),
-                             static_cast<uint64_t>(p.cand_idx[q]), q};
-                ++cnt;
+    if (p.sorted) {
+        // Runs of min(run_len, K) entries (a sorted run's entries past K never make
+        // the top-K); slot 0 holds the running result from the second chunk on.
+        const uint32_t rl = p.run_len;
+        const uint32_t nruns = (p.total + rl - 1) / rl;
+        const int use = rl < static_cast<uint32_t>(K) ? static_cast<int>(rl) : K;
+        const int slots = kMergeP / K;  // >= 2 (K <= 2048)
+        uint32_t next = 0;
+        bool first = true;
+        while (next < nruns) {
+            const int s0 = first ? 0 : 1;  // slot 0: the result so far (best first)
+            const uint32_t take = min(static_cast<uint32_t>(slots - s0), nruns - next);
+            const int used = s0 + static_cast<int>(take);
+            int P = 2 * K;
+            while (P < used * K) P <<= 1;
+            if (P < 64) P = 64;
+            // load: slot s = run next + s - s0, entries 0 .. use (odd slots reversed)
+            for (int q = tid; q < (P - s0 * K); q += kMergeNT) {
+                const int s = s0 + q / K, j = q % K;
+                const uint32_t r = next + static_cast<uint32_t>(s - s0);
+                EM e = EM::sentinel();
+                if (s < used && j < use) {
+                    const uint64_t g = static_cast<uint64_t>(r) * rl + j;
+                    if (g < p.total) e = entry(static_cast<uint32_t>(g));
+                }
+                b.st(s * K + ((s & 1) ? K - 1 - j : j), e);
             }
+            __syncthreads();
+            merge_net<CtaSync>(b, P, L, true, w, lane);
+            next += take;
+            first = false;
         }
-        int incl = cnt;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            int y = __shfl_up_sync(0xFFFFFFFFu, incl, o);
-            if (lane >= o) incl += y;
+    } else {
+        // General contract: any order.  Chunks of kMergeP - K new entries next to the
+        // running result, local sort + merge + rebuild.
+        uint32_t q0 = 0;
+        for (bool first = true; q0 < p.total; first = false) {
+            const int s0 = first ? 0 : K;
+            const int cnt = static_cast<int>(min(static_cast<uint32_t>(kMergeP - s0), p.total - q0));
+            int P = 2 * K;
+            while (P < s0 + cnt) P <<= 1;
+            if (P < 64) P = 64;
+            for (int i = tid; i < P - s0; i += kMergeNT)
+                b.st(s0 + i, i < cnt ? entry(q0 + static_cast<uint32_t>(i)) : EM::sentinel());
+            __syncthreads();
+            merge_net<CtaSync>(b, P, L, false, w, lane);
+            q0 += static_cast<uint32_t>(cnt);
         }
-        const int total = __shfl_sync(0xFFFFFFFFu, incl, 31);
-        int old = 0;
-        if (lane == 31 && total > 0) old = atomicAdd(&s_cnt, total);
-        old = __shfl_sync(0xFFFFFFFFu, old, 31);
-        int w = K + old + incl - cnt;
-#pragma unroll
-        for (int r = 0; r < CI; ++r)
-            if (q0 + tid + r * kMergeNT < p.total) buf.st(w++, ents[r]);
-        const int vote = (lane == 31 && old + total > flush_at) ? 1 : 0;
-        if (__syncthreads_or(vote)) do_flush();
     }
-    __syncthreads();
-    if (s_cnt > 0) do_flush();
     for (int j = tid; j < k; j += kMergeNT) {
-        const EM e = buf.ld(j);
+        const EM e = b.ld(j);
         if (p.out_idx) p.out_idx[j] = static_cast<int64_t>(e.idx);
         if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = ck[e.row];
         if (p.out_payload) p.out_payload[j] = p.cand_payload[e.row];

@@ -11,15 +11,9 @@ namespace {
 template <class Key, bool MIN>
 cudaError_t radix_seq(const RadixParams& p, cudaStream_t st) {
     using C = typename CodeOf<typename KeyTraits<Key>::E>::C;
-    static bool attr = false;
-    if (!attr) {
-        cudaError_t e = cudaFuncSetAttribute(radix_final<Key, MIN>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(kMergeSmem));
-        if (e != cudaSuccess) return e;
-
-        attr = true;
-    }
+    static std::atomic<uint64_t> attr{0};  // per device (dispatch.h)
+    const cudaError_t e = smem_attr_once(radix_final<Key, MIN>, static_cast<int>(kMergeSmem), attr);
+    if (e != cudaSuccess) return e;
     const int G = static_cast<int>(p.G);
     radix_hist<Key, MIN, true><<<G, kHistNT, 0, st>>>(p);
     radix_choose<C, true><<<1, kRadixBins, 0, st>>>(p);

@@ -423,23 +423,25 @@ __device__ __forceinline__ int append(const SBuf<E>& buf, int* s_cnt, const E (&
     return old;
 }
 
-// Debug counters (whole-launch totals), read with topk_debug_stats():
-// [0] flushes, [1] survivors flushed, [2] flush cycles (thread 0), [3] deferrals,
-// [4] tiles consumed, [5] refreshes, [6] exact flushes, [7] sentinel outputs (a bug).
-static __device__ unsigned long long g_stats[8];  // per translation unit (select_tu.cuh)
-
-// Debug timeline: per CTA up to 62 (event << 56 | globaltimer ns) stamps written by
-// consumer thread 0 (events: 1 start, 2 flush begin, 3 flush end, 4 stream end,
-// 5 tail begin, 6 end, 7 refresh); g_trace[c][0] = count.  Enabled by g_trace_on.
+// Debug instrumentation, compiled only into -DTOPK_DEBUG builds (tools/, variant
+// builds through _build.build(extra_flags=[...])); the product library has none of it.
+//  * g_stats: whole-launch counters read with topk_debug_stats(): [0] flushes,
+//    [1] survivors flushed, [2] flush cycles (thread 0), [3] deferrals, [4] tiles
+//    consumed, [5] refreshes, [6] exact flushes, [7] sentinel outputs (a bug).
+//  * g_trace: per CTA up to 62 (event << 56 | globaltimer ns) stamps written by consumer
+//    thread 0 (1 start, 2/3 flush begin/end, 4 stream end, 5 tail begin, 6 end,
+//    7 refresh); g_trace[c][0] = count.  Enabled by c_trace_on.
+//  * c_dbg: knobs (topk_debug_flags): bit 0 -- no code-network path; bit 1 -- no
+//    boot-time wait for peers; bit 2 -- no early second flush; bit 3 -- no small-buffer
+//    exact network; bits 4-5 -- rank-bound rows (0 = 3); bits 6-7 -- second-flush limit
+//    512 * (1 + v); bits 8-10 -- boot buffer kCap >> v (0 = by K).
 constexpr int kTraceCtas = 160, kTraceLen = 64;
+#ifdef TOPK_DEBUG
+static __device__ unsigned long long g_stats[8];  // per translation unit (select_inst.cuh)
 static __device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
-static __device__ __constant__ int c_trace_on;  // set by topk_debug_trace (constant bank: free)
-// Debug switches (topk_debug_flags): bit 0 -- no code-network path (exact flushes only);
-// bit 1 -- no boot-time wait for peers; bit 2 -- no early second flush; bit 3 -- no
-// small-buffer exact network (wnet_small); bits 4-5 -- rank-bound rows (0 = 3);
-// bits 6-7 -- second-flush limit 512 * (1 + v) (0 = TOPK_LIMIT2); bits 8-9 -- boot
-// buffer kCap >> v, bits 8-10 (0 = by K: 512 for K >= 256, else 4096).
+static __device__ __constant__ int c_trace_on;
 static __device__ __constant__ int c_dbg;
+#define TOPK_STAT(i, v) atomicAdd(&g_stats[i], static_cast<unsigned long long>(v))
 __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
     unsigned long long t;
@@ -451,6 +453,11 @@ __device__ __forceinline__ void trace(int ev) {
         row[0] = n + 1;
     }
 }
+#else
+constexpr int c_dbg = 0;
+#define TOPK_STAT(i, v) ((void)0)
+__device__ __forceinline__ void trace(int) {}
+#endif
 
 // Everything a collective needs besides the buffer.
 struct Ctx {
@@ -663,9 +670,9 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int c = static_cast<int>(blockIdx.x);
     int cnt = st->cnt;
-    const int cnt0 = cnt;
+    [[maybe_unused]] const int cnt0 = cnt;
     if (threadIdx.x == 0) trace(2);
-    const long long t0 = clock64();
+    [[maybe_unused]] const long long t0 = clock64();
     const bool publish = mode == kFlushStream && cx.filter;
     bool done = false;
     // (tie-heavy input -- a code bound cannot separate equal codes -- makes the code
@@ -722,10 +729,10 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         if (cnt > K) cnt = K;
     }
     if (threadIdx.x == 0) {
-        atomicAdd(&g_stats[0], 1ull);
-        atomicAdd(&g_stats[1], static_cast<unsigned long long>(cnt0));
-        atomicAdd(&g_stats[2], static_cast<unsigned long long>(clock64() - t0));
-        if (!done) atomicAdd(&g_stats[6], 1ull);
+        TOPK_STAT(0, 1ull);
+        TOPK_STAT(1, static_cast<unsigned long long>(cnt0));
+        TOPK_STAT(2, static_cast<unsigned long long>(clock64() - t0));
+        if (!done) TOPK_STAT(6, 1ull);
         if (tried && !done && publish) st->ties = 1;
         st->cnt = cnt;
         st->sorted_cnt = done ? -1 : cnt;
@@ -745,7 +752,7 @@ __device__ void refresh(CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx
     CSync::sync();
     rank_rows(st, cx);
     if (threadIdx.x == 0) {
-        atomicAdd(&g_stats[5], 1ull);
+        TOPK_STAT(5, 1ull);
         fold_bounds<Key, MIN>(st, cx, E::sentinel());
         st->req = 0;
         trace(7);
@@ -1270,7 +1277,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         int r = consume();
         while (r < 0) {  // did not fit: flush, then redo with the new bound
             if (lane == 0) {
-                atomicAdd(&g_stats[3], 1ull);
+                TOPK_STAT(3, 1ull);
                 atomicOr(&st.req, kReqFlush);
             }
             __syncwarp();
@@ -1288,7 +1295,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     while (cbar_or(pending_req())) collective();
     if (tid == 0) trace(4);
     if (tid == 0) {
-        atomicAdd(&g_stats[4], static_cast<unsigned long long>(ntiles_done));
+        TOPK_STAT(4, static_cast<unsigned long long>(ntiles_done));
         if (!st.pubd) atomicAdd(&hdr->npub, 1u);  // peers waiting at boot need not wait for us
     }
     // The CTA's run: the exact top-K of its bag, best first (skipped if already sorted).
@@ -1439,7 +1446,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     for (int j = tid; j < k; j += kNC) {
         const E e = buf.ld(j);
         if (e.is_sentinel()) {  // fewer than k rows (only a WHERE can do that, since k <= n)
-            if (Q == 0) atomicAdd(&g_stats[7], 1ull);  // plain form: a bug
+            if (Q == 0) TOPK_STAT(7, 1ull);  // plain form: a bug
             if (p.out_idx) p.out_idx[j] = -1;
             if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = Key{0};
             if constexpr ((Q & kQKey2) != 0)

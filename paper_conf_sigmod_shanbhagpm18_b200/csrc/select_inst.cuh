@@ -20,21 +20,23 @@ cudaError_t TOPK_INST_FN(const SelectParams& p, int grid, cudaStream_t st) {
     using Key = TOPK_INST_KEY;
     constexpr bool MIN = TOPK_INST_MIN, FILTER = TOPK_INST_FILTER;
     constexpr int Q = TOPK_INST_Q;
-    static std::atomic<bool> attr_set{false};  // idempotent
+    static std::atomic<uint64_t> attr_set{0};  // per device (dispatch.h)
     const size_t smem = select_smem_bytes<Key, Q>();
-    if (!attr_set.load(std::memory_order_relaxed)) {
-        cudaError_t e = cudaFuncSetAttribute(select_kernel<Key, MIN, FILTER, Q>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(smem));
-        if (e != cudaSuccess) return e;
-        attr_set.store(true, std::memory_order_relaxed);
-    }
+    const cudaError_t e =
+        smem_attr_once(select_kernel<Key, MIN, FILTER, Q>, static_cast<int>(smem), attr_set);
+    if (e != cudaSuccess) return e;
     select_kernel<Key, MIN, FILTER, Q><<<grid, kNT, smem, st>>>(p);
     return cudaGetLastError();
 }
 
 // This TU's copy of the debug globals (select.cuh g_stats, g_trace, c_dbg, c_trace_on).
 int TOPK_CAT(TOPK_INST_FN, _debug)(int op, void* host, int arg) {
+#ifndef TOPK_DEBUG
+    (void)op;
+    (void)host;
+    (void)arg;
+    return -1;  // debug globals exist only in -DTOPK_DEBUG builds
+#else
     switch (op) {
         case kDbgStatsAdd: {  // host: u64[8], accumulated
             unsigned long long v[8];
@@ -58,6 +60,7 @@ int TOPK_CAT(TOPK_INST_FN, _debug)(int op, void* host, int arg) {
         }
     }
     return -1;
+#endif
 }
 
 }  // namespace topk

@@ -147,8 +147,8 @@ topk_status_t topk_select_sharded(topk_dtype_t dtype, const void* keys, const ui
     // (3) the global step: exact top-k of the G sorted candidate runs
     return merge_total(dtype, w + L.gk, reinterpret_cast<const int64_t*>(w + L.gi),
                        payload ? reinterpret_cast<const uint32_t*>(w + L.gp) : nullptr,
-                       static_cast<uint64_t>(nranks) * k, k, order, out_keys, out_payload, out_idx,
-                       stream);
+                       static_cast<uint64_t>(nranks) * k, k, true, k, order, out_keys,
+                       out_payload, out_idx, stream);
 }
 
 topk_status_t topk_f32_sharded(const float* keys, uint64_t n_local, uint64_t base, uint32_t k,

@@ -10,7 +10,6 @@
 
 #include "merge.cuh"
 #include "probe.cuh"
-#include "netbench.cuh"
 #include "dispatch.h"
 #include "radix.cuh"
 #include "select.cuh"
@@ -85,14 +84,10 @@ int key_kind(topk_dtype_t dt) {
 
 template <class Key, bool MIN>
 cudaError_t launch_merge(const topk::MergeParams& p, cudaStream_t st) {
-    static bool attr_set = false;
-    if (!attr_set) {
-        cudaError_t e = cudaFuncSetAttribute(topk::merge_kernel<Key, MIN>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             static_cast<int>(topk::kMergeSmem));
-        if (e != cudaSuccess) return e;
-        attr_set = true;
-    }
+    static std::atomic<uint64_t> attr_set{0};  // per device (dispatch.h)
+    const cudaError_t e = topk::smem_attr_once(topk::merge_kernel<Key, MIN>,
+                                               static_cast<int>(topk::kMergeSmem), attr_set);
+    if (e != cudaSuccess) return e;
     topk::merge_kernel<Key, MIN><<<1, topk::kMergeNT, topk::kMergeSmem, st>>>(p);
     g_launches.fetch_add(1, std::memory_order_relaxed);
     return cudaGetLastError();
@@ -146,10 +141,13 @@ size_t select_ws_bytes(topk_dtype_t dtype, uint32_t k, int sms) {
 }  // namespace
 
 // Merge `total` candidate entries (contiguous) to the exact top-k (topk_merge's body).
+// run_len: entries per run (the last run may be shorter); sorted: every run is sorted
+// best first (topk_select's output), so the merge kernel skips the local sort.
 static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
                                  const int64_t* cand_idx, const uint32_t* cand_payload,
-                                 uint64_t total, uint32_t k, topk_order_t order, void* out_keys,
-                                 uint32_t* out_payload, int64_t* out_idx, void* stream);
+                                 uint64_t total, uint32_t run_len, bool sorted, uint32_t k,
+                                 topk_order_t order, void* out_keys, uint32_t* out_payload,
+                                 int64_t* out_idx, void* stream);
 // chunked-input helpers (used by topk_workspace_bytes / topk_select).  Chunk length
 // 2^31 keys; TOPK_CHUNK_N (multiple of 4) overrides it so tests can exercise the
 // chunked path on small inputs.
@@ -272,7 +270,6 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
     // default: one block per SM per wave -- all SMs stream one address window at a
     // time (DRAM row locality), waves in pseudo-random order (robust to sorted input)
     p.wave = wave_env > 0 ? static_cast<uint32_t>(wave_env) : static_cast<uint32_t>(sms);
-    if (false) p.wave = wave_env > 0 ? static_cast<uint32_t>(wave_env) : 1u;
     p.nwaves = (p.nblocks + p.wave - 1) / p.wave;
     uint32_t bits = 0;
     while ((1ull << bits) < p.nwaves) ++bits;
@@ -316,13 +313,21 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
     if (n <= kMaxLaunchN && n <= chunk_n())
         return select_one(dtype, keys, payload, n, base, k, order, mode, out_keys, out_payload,
                           out_idx, ws, ws_bytes, stream);
-    if (!valid_dtype(dtype) || !keys || k == 0 || k > TOPK_MAX_K) return TOPK_ERR_INVALID_ARG;
+    // every argument error is reported before the first chunk is enqueued
+    if (!valid_dtype(dtype) || !valid_order(order) || !keys || k == 0 || k > TOPK_MAX_K ||
+        k > n)
+        return TOPK_ERR_INVALID_ARG;
+    if (mode != TOPK_MODE_FILTER && mode != TOPK_MODE_PURE) return TOPK_ERR_INVALID_ARG;
+    if (out_payload && !payload) return TOPK_ERR_INVALID_ARG;
+    if (reinterpret_cast<uintptr_t>(keys) % key_size(dtype)) return TOPK_ERR_INVALID_ARG;
     int sms = 0, major = 0;
     if (!device_info(&sms, &major)) return TOPK_ERR_CUDA;
+    if (major != 10 || sms > topk::kGMax) return TOPK_ERR_UNSUPPORTED;
     const uint64_t nch = (n + chunk_n() - 1) / chunk_n();
     if (nch * k > 65536) return TOPK_ERR_UNSUPPORTED;
     const ChunkLayout L = chunk_layout(dtype, nch, k, sms);
-    if (!ws || ws_bytes < L.total) return TOPK_ERR_WORKSPACE;
+    if (!ws || ws_bytes < L.total || (reinterpret_cast<uintptr_t>(ws) % 256))
+        return TOPK_ERR_WORKSPACE;
     unsigned char* w = static_cast<unsigned char*>(ws);
     const size_t ks = key_size(dtype);
     uint64_t total = 0;
@@ -337,9 +342,10 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
         if (st != TOPK_OK) return st;
         total += kc;
     }
+    // the chunks' results are sorted runs of k entries (the last one may be shorter)
     return merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
                        payload ? reinterpret_cast<const uint32_t*>(w + L.cp) : nullptr, total, k,
-                       order, out_keys, out_payload, out_idx, stream);
+                       true, k, order, out_keys, out_payload, out_idx, stream);
 }
 
 topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank_b,
@@ -543,8 +549,21 @@ topk_status_t topk_merge(topk_dtype_t dtype, const void* cand_keys, const int64_
     (void)ws_bytes;
     if (runs == 0 || run_len == 0) return TOPK_ERR_INVALID_ARG;
     return merge_total(dtype, cand_keys, cand_idx, cand_payload,
-                       static_cast<uint64_t>(runs) * run_len, k, order, out_keys, out_payload,
-                       out_idx, stream);
+                       static_cast<uint64_t>(runs) * run_len, run_len, false, k, order, out_keys,
+                       out_payload, out_idx, stream);
+}
+
+topk_status_t topk_merge_sorted(topk_dtype_t dtype, const void* cand_keys,
+                                const int64_t* cand_idx, const uint32_t* cand_payload,
+                                uint32_t runs, uint32_t run_len, uint32_t k, topk_order_t order,
+                                void* out_keys, uint32_t* out_payload, int64_t* out_idx,
+                                void* ws, size_t ws_bytes, void* stream) {
+    (void)ws;
+    (void)ws_bytes;
+    if (runs == 0 || run_len == 0) return TOPK_ERR_INVALID_ARG;
+    return merge_total(dtype, cand_keys, cand_idx, cand_payload,
+                       static_cast<uint64_t>(runs) * run_len, run_len, true, k, order, out_keys,
+                       out_payload, out_idx, stream);
 }
 
 /* Debug (not in topk.h's stable surface): read / reset the device counters of
@@ -585,26 +604,6 @@ topk_status_t topk_probe_read(const void* data, size_t bytes, int method, int gr
     }
     g_launches.fetch_add(1, std::memory_order_relaxed);
     return cudaGetLastError() == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
-}
-
-/* Debug: cycles of one flush network call on P entries (K = 2^L), measured in one CTA
- * of 15 warps.  e64 selects 12-byte entries; smem_net the shared-memory network. */
-int topk_debug_netbench(int P, int L, int e64, int smem_net, int iters, uint64_t* host2) {
-    unsigned long long* d = nullptr;
-    if (cudaMalloc(&d, 24) != cudaSuccess) return -1;
-    const size_t smem = 4096 * 12 + 4096 * 8;
-    if (e64) {
-        cudaFuncSetAttribute(topk::netbench_kernel<topk::E64, 15>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        topk::netbench_kernel<topk::E64, 15><<<1, 480, smem>>>(P, L, iters, smem_net, d);
-    } else {
-        cudaFuncSetAttribute(topk::netbench_kernel<topk::E32, 15>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        topk::netbench_kernel<topk::E32, 15><<<1, 480, smem>>>(P, L, iters, smem_net, d);
-    }
-    cudaError_t e = cudaMemcpy(host2, d, 16, cudaMemcpyDeviceToHost);
-    cudaFree(d);
-    return e == cudaSuccess ? 0 : -1;
 }
 
 /* Debug: the code-only network (cnet.cuh) on n <= 4096 device codes (u32, or u64 if
@@ -739,7 +738,7 @@ topk_status_t topk_select_host(topk_dtype_t dtype, const void* h_keys, uint64_t 
         total += kc;
     }
     topk_status_t r = merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
-                                  nullptr, total, k, order, w + L.ok, nullptr,
+                                  nullptr, total, k, true, k, order, w + L.ok, nullptr,
                                   reinterpret_cast<int64_t*>(w + L.oi), stream);
     if (r != TOPK_OK) return r;
     if (h_out_keys &&
@@ -771,8 +770,9 @@ int topk_abi_version(void) { return TOPK_ABI_VERSION; }
 
 static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
                                  const int64_t* cand_idx, const uint32_t* cand_payload,
-                                 uint64_t total, uint32_t k, topk_order_t order, void* out_keys,
-                                 uint32_t* out_payload, int64_t* out_idx, void* stream) {
+                                 uint64_t total, uint32_t run_len, bool sorted, uint32_t k,
+                                 topk_order_t order, void* out_keys, uint32_t* out_payload,
+                                 int64_t* out_idx, void* stream) {
     if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
     if (!cand_keys || !cand_idx || total == 0) return TOPK_ERR_INVALID_ARG;
     if (total > 65536 || k == 0 || k > TOPK_MAX_K || k > total) return TOPK_ERR_INVALID_ARG;
@@ -788,6 +788,8 @@ static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
     p.out_payload = out_payload;
     p.out_idx = out_idx;
     p.total = static_cast<uint32_t>(total);
+    p.run_len = run_len == 0 ? 1u : run_len;
+    p.sorted = sorted ? 1u : 0u;
     p.k = k;
     p.K = next_pow2_u32(k);
     cudaStream_t st = static_cast<cudaStream_t>(stream);

@@ -25,9 +25,6 @@
 
 namespace topk {
 
-// netbench instrumentation: clock64 at the end of phase A of the last network call
-static __device__ long long g_wnet_phase_a_end;  // per translation unit
-
 template <class E>
 __device__ __forceinline__ E shfl_xor_e(const E& e, int m);
 template <>
@@ -224,7 +221,6 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
         }
     }
     Sync::sync();
-    if (threadIdx.x == 0) g_wnet_phase_a_end = clock64();
     // local-sort stages beyond 512-runs (len 512, 1024): bits >= 9 in smem, 8..0 in registers
 #pragma unroll 1
     for (int d = 10; d <= L; ++d) {
@@ -382,8 +378,12 @@ __device__ __forceinline__ void wsmall_step(E (&x)[R], const SBuf<E>& b, int P, 
     }
 }
 
+// presorted: b already holds runs of 2^L alternating best-first / worst-first (the state
+// the local sort leaves) -- only the merge + rebuild rounds run (the merge kernel's
+// sorted candidate runs).
 template <class E, int R, int NW, class Sync>
-__device__ void wnet_small(const SBuf<E>& b, int P, int L, int w, int lane) {
+__device__ void wnet_small(const SBuf<E>& b, int P, int L, int w, int lane,
+                           bool presorted = false) {
     const int W = P / (32 * R);
     const bool act = w < W;
     const uint32_t e0 = static_cast<uint32_t>(w * 32 * R + lane * R);
@@ -396,7 +396,7 @@ __device__ void wnet_small(const SBuf<E>& b, int P, int L, int w, int lane) {
     }
     int region = 1;
 #pragma unroll 1
-    for (int s = 0; s < L; ++s)
+    for (int s = 0; s < (presorted ? 0 : L); ++s)
 #pragma unroll 1
         for (int bb = s; bb >= 0; --bb)
             wsmall_step<E, R, Sync>(x, b, P, e0, lane, act, bb, s + 1, region);

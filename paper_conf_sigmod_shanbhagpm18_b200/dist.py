@@ -110,24 +110,30 @@ def sharded_topk_native(x_local: torch.Tensor, k: int, comm: NcclComm, largest: 
     merge kernel, all enqueued on the current stream (no host synchronisation).
     Returns (values, int64 global ids[, payload]) on every rank."""
     import ctypes
-    from . import _lib, _dtype_code, _ptr, _stream_ptr
+    from . import _lib, _dtype_code, _ptr, _stream_ptr, _check_col, _check_out
     if not x_local.is_cuda or x_local.dim() != 1:
         raise ValueError("sharded_topk_native expects a 1-D CUDA tensor")
+    if x_local.device != comm.device:
+        raise ValueError(f"shard on {x_local.device}, communicator on {comm.device}")
     lib = _lib.load()
     dt = _dtype_code(x_local)
     n = x_local.shape[0]
+    dev = x_local.device
     x_local = x_local.contiguous()
+    payload = _check_col(payload, n, torch.uint32, dev, "payload")
     if out is None:
-        vals = torch.empty(k, dtype=x_local.dtype, device=x_local.device)
-        idx = torch.empty(k, dtype=torch.int64, device=x_local.device)
-        pay = torch.empty(k, dtype=torch.uint32, device=x_local.device) \
-            if payload is not None else None
+        vals = torch.empty(k, dtype=x_local.dtype, device=dev)
+        idx = torch.empty(k, dtype=torch.int64, device=dev)
+        pay = torch.empty(k, dtype=torch.uint32, device=dev) if payload is not None else None
     else:
-        vals, idx, pay = out
-    ws = comm.workspace(dt, n, k)
-    st = lib.topk_select_sharded(dt, _ptr(x_local), _ptr(payload), n, base, k,
-                                 _lib.LARGEST if largest else _lib.SMALLEST, _ptr(vals),
-                                 _ptr(pay), _ptr(idx), comm.ptr, ws.ptr(), ws.nbytes,
-                                 _stream_ptr(x_local.device))
+        vals = _check_out(out[0], k, x_local.dtype, dev, "out values")
+        idx = _check_out(out[1], k, torch.int64, dev, "out indices")
+        pay = _check_out(out[2], k, torch.uint32, dev, "out payload")
+    with torch.cuda.device(dev):
+        ws = comm.workspace(dt, n, k)
+        st = lib.topk_select_sharded(dt, _ptr(x_local), _ptr(payload), n, base, k,
+                                     _lib.LARGEST if largest else _lib.SMALLEST, _ptr(vals),
+                                     _ptr(pay), _ptr(idx), comm.ptr, ws.ptr(), ws.nbytes,
+                                     _stream_ptr(dev))
     _lib.check(st, "topk_select_sharded")
     return (vals, idx) if payload is None else (vals, idx, pay)

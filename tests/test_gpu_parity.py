@@ -127,16 +127,47 @@ def test_base_offset(cuda_device):
 
 def test_merge_kernel(cuda_device):
     rng = np.random.default_rng(4)
-    for runs, run_len, k in [(8, 256, 256), (4, 1024, 1000), (3, 5, 7), (16, 64, 64)]:
+    for runs, run_len, k in [(8, 256, 256), (4, 1024, 1000), (3, 5, 7), (16, 64, 64),
+                             (1, 9000, 2048), (64, 1024, 1), (30, 2000, 500)]:
         vals = rng.choice(np.array([0.5, 1.0, np.nan, -0.0, 0.0, 2.0], np.float32),
                           runs * run_len)
-        idx = rng.permutation(10 ** 9)[: runs * run_len].astype(np.int64)
+        idx = rng.choice(10 ** 9, size=runs * run_len, replace=False).astype(np.int64)
         for largest in (True, False):
             v, i = tk.merge(torch.from_numpy(vals).cuda(), torch.from_numpy(idx).cuda(), k,
                             largest, runs=runs)
             ov, oi = oracle.topk(vals, k, largest, idx=idx)
             assert np.array_equal(i.cpu().numpy(), oi)
             assert v.cpu().numpy().tobytes() == ov.tobytes()
+
+
+@pytest.mark.parametrize("runs,run_len,k", [(8, 256, 256), (2, 256, 256), (8, 1024, 1024),
+                                            (4, 2048, 2048), (64, 256, 256), (3, 100, 77),
+                                            (5, 300, 64), (16, 64, 1), (1, 512, 500),
+                                            (32, 2048, 2048)])
+@pytest.mark.parametrize("largest", [True, False])
+def test_merge_sorted_runs(cuda_device, runs, run_len, k, largest):
+    """topk_merge_sorted: runs sorted best first (each the oracle's top-run_len of a
+    random tie-heavy block with distinct global ids) -> merge + rebuild rounds only;
+    result == the oracle's top-k of all candidates."""
+    rng = np.random.default_rng(runs * 1000 + run_len + k)
+    vals, idxs = [], []
+    pool = np.array([0.5, 1.0, np.nan, -0.0, 0.0, 2.0, -1.0, np.inf], np.float32)
+    gids = rng.choice(10 ** 9, size=runs * run_len * 2, replace=False).astype(np.int64).reshape(runs, -1)
+    for r in range(runs):
+        block = rng.choice(pool, 2 * run_len)
+        v, i = oracle.topk(block, run_len, largest, idx=gids[r])
+        vals.append(v)
+        idxs.append(i)
+    cv, ci = np.concatenate(vals), np.concatenate(idxs)
+    pay = rng.integers(0, 2 ** 32, cv.shape[0], dtype=np.uint64).astype(np.uint32)
+    v, i, pv = tk.merge(torch.from_numpy(cv).cuda(), torch.from_numpy(ci).cuda(), k, largest,
+                        cand_payload=torch.from_numpy(pay.view(np.int32)).cuda().view(torch.uint32),
+                        runs=runs, sorted_runs=True)
+    ov, oi = oracle.topk(cv, k, largest, idx=ci)
+    assert np.array_equal(i.cpu().numpy(), oi)
+    assert v.cpu().numpy().tobytes() == ov.tobytes()
+    row = {int(g): j for j, g in enumerate(ci)}
+    assert np.array_equal(host(pv), pay[[row[int(g)] for g in oi]])
 
 
 def test_sharded_on_one_gpu(cuda_device):
@@ -152,9 +183,12 @@ def test_sharded_on_one_gpu(cuda_device):
             v, i = tk.topk(xd[cuts[r]:cuts[r + 1]], k, True, base=cuts[r])
             vs.append(v)
             is_.append(i)
-        mv, mi = tk.merge(torch.cat(vs), torch.cat(is_), k, True, runs=G)
         ov, oi = oracle.topk(x.numpy(), k, True)
-        assert np.array_equal(mi.cpu().numpy(), oi)
+        for sorted_runs in (False, True):
+            mv, mi = tk.merge(torch.cat(vs), torch.cat(is_), k, True, runs=G,
+                              sorted_runs=sorted_runs)
+            assert np.array_equal(mi.cpu().numpy(), oi)
+            assert mv.cpu().numpy().tobytes() == ov.tobytes()
 
 
 def test_repeated_calls_reuse_workspace(cuda_device):

@@ -260,8 +260,12 @@ def test_three_keys(cuda_device, orders):
 
 
 def test_three_keys_full_ties_predicate_payload(cuda_device):
-    cols = [datagen.generate("fewdistinct", N, "f32", seed=334) for _ in range(3)]
-    run_kkk(cols, 500, (True, True, False))  # 16^3 distinct tuples: the row id decides
+    # three independent 16-value columns: 16^3 = 4096 distinct tuples over N rows, so
+    # every tuple repeats and key 2 / key 3 / the row id all decide somewhere
+    cols = [datagen.generate("fewdistinct", N, "f32", seed=334 + 10 * j) for j in range(3)]
+    h = [c.numpy() for c in cols]
+    assert len({(a, b) for a, b in zip(h[0][:4096], h[1][:4096])}) > 16  # columns differ
+    run_kkk(cols, 500, (True, True, False))
     col = u32col(N, 335, 10)
     pay = datagen.payload(N, seed=336)
     run_kkk(cols, 64, (False, False, True), pred=("range", col, 3, 8), payload=pay)

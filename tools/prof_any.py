@@ -1,6 +1,6 @@
 """Run one hot-path op a few times (for an ncu capture of its kernel; dev tool).
 
-    python tools/prof_any.py select|query1|query2|kk|kkk|radix K
+    python tools/prof_any.py select|pure|query1|query2|kk|kkk|radix K
 """
 import os
 import sys
@@ -13,9 +13,10 @@ from paper_conf_sigmod_shanbhagpm18_b200 import datagen
 
 op, k = sys.argv[1], int(sys.argv[2])
 dev = "cuda"
-if op in ("select", "radix"):
+if op in ("select", "radix", "pure"):
     x = datagen.generate("uniform", 1 << 29, "f32", seed=datagen.config_seed(2), device=dev)
-    f = (lambda: tk.topk(x, k)) if op == "select" else (lambda: tk.topk_radix(x, k))
+    f = {"select": lambda: tk.topk(x, k), "radix": lambda: tk.topk_radix(x, k),
+         "pure": lambda: tk.topk(x, k, mode="pure")}[op]
 elif op == "query1":
     n = 1 << 28
     cnt = datagen.generate("uniform", n, "u32", seed=datagen.config_seed(6), device=dev)

@@ -33,6 +33,13 @@ KEYS = [
     "smsp__sass_average_branch_targets_threads_uniform.pct",
     "sm__inst_executed_pipe_alu.avg.pct_of_peak_sustained_active",
     "sm__cycles_elapsed.avg.per_second", "lts__t_bytes.sum",
+    "sm__issue_active.avg.pct_of_peak_sustained_elapsed",
+    "sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active",
+    "sm__inst_executed_pipe_fma.avg.pct_of_peak_sustained_active",
+    "smsp__average_warps_issue_stalled_barrier_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_short_scoreboard_per_issue_active.ratio",
+    "smsp__average_warps_issue_stalled_wait_per_issue_active.ratio",
 ]
 
 
