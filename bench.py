@@ -249,7 +249,8 @@ def ncu_traffic(k, n, timeout=420):
     h = rows[0]
     ni, vi, ui = h.index("Metric Name"), h.index("Metric Value"), h.index("Metric Unit")
     scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
-             "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3, "second": 1.0}
+             "nsecond": 1e-9, "usecond": 1e-6, "msecond": 1e-3, "second": 1.0,
+             "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "s": 1.0}
     m = {row[ni]: float(row[vi].replace(",", "")) * scale.get(row[ui], 1.0) for row in rows[1:]}
     rd, wr = m.get("dram__bytes_read.sum"), m.get("dram__bytes_write.sum")
     if rd is None or wr is None:
@@ -273,9 +274,21 @@ def run_ncu_target(args):
 def size_sweep(tk, datagen, stream, torch, peak, k=64):
     """Fig. 13: data size 2^21 ... 2^29 uniform f32 at fixed k = 64.  Inputs
     that fit the 126 MB L2 (<= 2^25 keys) are timed one launch at a time with the L2
-    flushed before each launch (a 512 MiB write); larger ones back to back."""
+    flushed before each launch (a read of 512 MiB, which leaves clean lines -- a write
+    would leave dirty lines whose write-back lands inside the timed launch); larger ones
+    back to back."""
+    import ctypes
+    from paper_conf_sigmod_shanbhagpm18_b200 import _lib
+    lib = _lib.load()
     dev = stream.device
-    scrub = torch.empty(1 << 27, dtype=torch.int32, device=dev)
+    scrub = torch.ones(1 << 27, dtype=torch.int32, device=dev)
+    sink = torch.zeros(4, dtype=torch.int32, device=dev)
+
+    def flush_l2():
+        _lib.check(lib.topk_probe_read(ctypes.c_void_p(scrub.data_ptr()), scrub.numel() * 4, 0, 0,
+                                       0, 0, ctypes.c_void_p(sink.data_ptr()),
+                                       ctypes.c_void_p(stream.cuda_stream)), "probe (L2 flush)")
+
     out = []
     for lg in range(21, 30):
         n = 1 << lg
@@ -287,7 +300,7 @@ def size_sweep(tk, datagen, stream, torch, peak, k=64):
         if lg <= 25:
             per = []
             for _ in range(10):
-                scrub.zero_()
+                flush_l2()
                 _, t = time_steps(f, 1, stream, torch, per_step=True)
                 per.append(t[0])
             us = statistics.median(per) * 1e3
@@ -494,6 +507,7 @@ def run_extras(args, tk, datagen, x, stream, torch, hbm):
     t = timed(lambda: tk.topk(x1, 32, True), 50)
     cfgs.append({"config": "BJ1: 2^20 uniform f32, k=32 (launch-bound, L2-resident, back to back)",
                  "us": round(t * 1e3, 2), "keys_per_s": (1 << 20) / (t / 1e3)})
+    x1 = None
     del x1
     n4 = 1 << 28
     xu = datagen.generate("uniform", n4, "u32", seed=datagen.config_seed(4), device=dev)

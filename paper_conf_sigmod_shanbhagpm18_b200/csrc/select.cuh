@@ -446,11 +446,15 @@ __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    // (the event count lives in shared memory: a stamp costs one fire-and-forget store)
     unsigned long long* row = g_trace[blockIdx.x];
-    const unsigned long long n = row[0];
+    __shared__ int s_trace_n;
+    if (ev == 1) s_trace_n = 0;
+    const int n = s_trace_n;
     if (n + 1 < kTraceLen) {
         row[n + 1] = (static_cast<unsigned long long>(ev) << 56) | (t & 0x00FFFFFFFFFFFFFFull);
-        row[0] = n + 1;
+        row[0] = static_cast<unsigned long long>(n + 1);
+        s_trace_n = n + 1;
     }
 }
 #else

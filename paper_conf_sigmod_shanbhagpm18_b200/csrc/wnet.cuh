@@ -341,8 +341,14 @@ __device__ __forceinline__ void wsmall_step(E (&x)[R], const SBuf<E>& b, int P, 
     if (bb < LR) {
         if (!act) return;
         // compile-time register pairs (a runtime index would put x in local memory)
-        if (bb == 0) wsmall_reg<E, R, 0>(x, e0, d);
-        else if constexpr (LR > 1) wsmall_reg<E, R, 1>(x, e0, d);
+        if (bb == 0) {
+            wsmall_reg<E, R, 0>(x, e0, d);
+        } else if (bb == 1) {
+            if constexpr (LR > 1) wsmall_reg<E, R, 1>(x, e0, d);
+        } else {
+            if constexpr (LR > 2) wsmall_reg<E, R, 2>(x, e0, d);
+        }
+        static_assert(LR <= 3, "wnet_small: at most 8 entries per lane");
     } else if (bb < LR + 5) {
         if (!act) return;
         const int m = 1 << (bb - LR);

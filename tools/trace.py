@@ -20,7 +20,8 @@ for c in range(148):
     m = int(buf[c, 0]); ev = [(int(v) >> 56, int(v) & ((1 << 56) - 1)) for v in buf[c, 1:m + 1]]
     if ev: rows.append(ev)
 t0 = min(e[0][1] for e in rows)
-names = {1: "start", 2: "fb", 3: "fe", 4: "sEnd", 5: "tail", 6: "end", 7: "refr", 8: "sampled", 9: "ranked", 10: "appended", 11: "tb", 12: "ph0", 13: "ph1", 14: "loaded", 15: "apd"}
+names = {1: "start", 2: "fb", 3: "fe", 4: "sEnd", 5: "tail", 6: "end", 7: "refr", 8: "sampled", 9: "ranked", 10: "appended", 11: "tb", 12: "ph0", 13: "ph1", 14: "loaded", 15: "apd",
+         16: "cnet", 17: "bnd", 18: "cmp", 19: "wnet", 20: "wait", 21: "lpub", 22: "rank"}
 send_c = [(max([t for e, t in ev if e == 4] or [0]), c) for c, ev in enumerate(rows)]
 send_c.sort()
 for _, c in send_c[:2] + send_c[-3:]:
@@ -40,3 +41,4 @@ print(json.dumps(dict(k=k, dist=dist, flushes_per_cta=float(np.mean(fl)), flush_
 # histogram of flush begin times
 hb = np.histogram([b / 1000 for b, _ in ft], bins=10)
 print("flush begin hist (us):", [f"{e:.0f}:{c}" for c, e in zip(hb[0], hb[1])])
+
