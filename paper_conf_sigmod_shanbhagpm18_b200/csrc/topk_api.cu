@@ -11,6 +11,7 @@
 #include "merge.cuh"
 #include "probe.cuh"
 #include "dispatch.h"
+#include "pure.cuh"
 #include "radix.cuh"
 #include "select.cuh"
 #include "topk.h"
@@ -132,9 +133,11 @@ uint32_t query_tile_keys(topk_dtype_t dt, int q) {
     }
 }
 
+// Candidate area: one run of next_pow2(k) entries per CTA (the pure-mode kernel keeps
+// whole K-runs; the streaming select keeps k).
 size_t select_ws_bytes(topk_dtype_t dtype, uint32_t k, int sms) {
     return align_up(topk::ws_cand_offset(static_cast<uint32_t>(sms)) +
-                        static_cast<size_t>(sms) * k * entry_bytes(dtype),
+                        static_cast<size_t>(sms) * next_pow2_u32(k) * entry_bytes(dtype),
                     256);
 }
 
@@ -287,6 +290,27 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
+    if (!filt && !qa.q && dtype != TOPK_F64 && p.K <= 32) {
+        // the paper's pure method, register/shuffle form (pure.cuh): 32-bit keys, K <= 32
+        topk::PureParams pp;
+        pp.keys = keys;
+        pp.payload = payload;
+        pp.out_keys = out_keys;
+        pp.out_payload = out_payload;
+        pp.out_idx = out_idx;
+        pp.ticket = reinterpret_cast<unsigned int*>(p.ws) + 5;  // WsHeader::pad[0]
+        pp.cand = reinterpret_cast<uint64_t*>(p.ws + topk::ws_cand_offset(p.gmax));
+        pp.n = n;
+        pp.base = base;
+        pp.k = k;
+        pp.L = static_cast<uint32_t>(__builtin_ctz(p.K));
+        const uint64_t nch = (n + topk::kPureChunk - 1) / topk::kPureChunk;
+        const uint64_t want = (nch + topk::kPureNW - 1) / topk::kPureNW;  // one chunk per warp
+        const int pgrid = static_cast<int>(want < static_cast<uint64_t>(sms) ? want : sms);
+        const cudaError_t e = topk::launch_pure(key_kind(dtype), mn, pp, pgrid, st);
+        if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
+        return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
+    }
     if (qa.q & topk::kQKey2) {
         p.out_keys2 = qa.out_keys2;
         p.order2_min = qa.order2_min;
