@@ -213,6 +213,9 @@ __device__ __forceinline__ void warp_append(RadixEntry<C>* list, uint32_t* cnt, 
 // per warp in shared memory, fire-and-forget shared atomics (no result is waited for,
 // so a thread's 16 increments pipeline; same-bin lanes serialise in the atomic unit --
 // U(0,1) floats put half the keys on one first digit), warps summed at the end.
+#ifndef TOPK_RADIX_MATCH
+#define TOPK_RADIX_MATCH 0
+#endif
 constexpr int kHistNT = 256;
 constexpr size_t kHistSmem = size_t(kHistNT / 32) * kRadixBins * sizeof(uint32_t);  // 8 KB
 template <class Key, bool MIN, bool FIRST>
@@ -242,9 +245,18 @@ __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
             const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
             load_codes<Key, MIN>(keys, hi, r0, c);
 #pragma unroll
-            for (int q = 0; q < kRadixPerThread; ++q)
-                if (r0 + q < hi && has_prefix(c[q], prefix, shift))
-                    atomicAdd(&mine[digit_of(c[q], shift)], 1u);
+            for (int q = 0; q < kRadixPerThread; ++q) {
+                const bool ok = r0 + q < hi && has_prefix(c[q], prefix, shift);
+#if TOPK_RADIX_MATCH
+                // lanes with the same digit add once (U(0,1) floats put half the keys on
+                // one first digit: same-address shared atomics would serialise)
+                const uint32_t d = ok ? digit_of(c[q], shift) : 0x100u + (threadIdx.x & 31);
+                const uint32_t peers = __match_any_sync(0xFFFFFFFFu, d);
+                if (ok && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(&mine[d], __popc(peers));
+#else
+                if (ok) atomicAdd(&mine[digit_of(c[q], shift)], 1u);
+#endif
+            }
         }
     }
     __syncthreads();
@@ -319,20 +331,20 @@ __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
     if (!w.st->scatter) return;
     const uint32_t kTop = w.st->bshift;
     const C d1 = w.st->prefix >> kTop;
-    // bucket entries are staged in shared memory and written with one global
-    // reservation per flush (a per-warp atomic on one counter serialises in L2)
-    constexpr int kStage = 2048;
-    __shared__ RadixEntry<C> stage[kStage];
-    __shared__ uint32_t s_w[kRadixNT / 32];
-    __shared__ uint32_t s_base;
-    uint32_t staged = 0;
-    auto flush = [&]() {
-        if (threadIdx.x == 0) s_base = atomicAdd(&w.st->nbucket, staged);
-        __syncthreads();
-        const uint32_t base = s_base;
-        for (uint32_t i = threadIdx.x; i < staged; i += kRadixNT)
-            if (base + i < p.cap) w.bucket[base + i] = stage[i];
-        __syncthreads();
+    // bucket entries are staged per warp in shared memory (warp-aggregated appends, no
+    // CTA barrier) and written with one global reservation per warp flush
+    constexpr int kWStage = 256;
+    __shared__ RadixEntry<C> stage[kRadixNT / 32][kWStage];
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t lt = (1u << lane) - 1u;
+    uint32_t staged = 0;  // warp-uniform
+    auto wflush = [&]() {
+        uint32_t base = 0;
+        if (lane == 0) base = atomicAdd(&w.st->nbucket, staged);
+        base = __shfl_sync(0xFFFFFFFFu, base, 0);
+        for (uint32_t i = lane; i < staged; i += 32)
+            if (base + i < p.cap) w.bucket[base + i] = stage[warp][i];
+        __syncwarp();
         staged = 0;
     };
     const Key* keys = static_cast<const Key*>(p.keys);
@@ -341,13 +353,20 @@ __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
         C c[kRadixPerThread];
         const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
         load_codes<Key, MIN>(keys, hi, r0, c);
-        uint32_t nb = 0, gtm = 0;
+        uint32_t gtm = 0;
 #pragma unroll
         for (int q = 0; q < kRadixPerThread; ++q) {
             const bool ok = r0 + q < hi;
             const C dg = c[q] >> kTop;  // code above the bucket's bits
-            nb += (ok && dg == d1) ? 1u : 0u;
             gtm |= static_cast<uint32_t>(ok && dg > d1) << q;
+            const bool in = ok && dg == d1;
+            const uint32_t m = __ballot_sync(0xFFFFFFFFu, in);
+            if (m) {
+                if (staged + __popc(m) > kWStage) wflush();
+                if (in) stage[warp][staged + __popc(m & lt)] =
+                            RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)};
+                staged += __popc(m);
+            }
         }
         // entries above the bucket: fewer than k in all (rare: one vote per tile, then
         // warp-aggregated appends)
@@ -357,32 +376,9 @@ __global__ void __launch_bounds__(kRadixNT) radix_scatter(const RadixParams p) {
                 warp_append(w.gt, &w.st->ngt, p.k, (gtm >> q) & 1u,
                             RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)}, nullptr);
         }
-        uint32_t tile_nb;
-        const uint32_t off = block_excl_scan(nb, s_w, &tile_nb);
-        if (tile_nb == 0) continue;
-        if (staged + tile_nb > kStage) flush();
-        if (tile_nb > kStage) {  // a tile mostly in the bucket (e.g. sorted input): direct
-            if (threadIdx.x == 0) s_base = atomicAdd(&w.st->nbucket, tile_nb);
-            __syncthreads();
-            uint32_t at = s_base + off;
-#pragma unroll
-            for (int q = 0; q < kRadixPerThread; ++q)
-                if (r0 + q < hi && (c[q] >> kTop) == d1) {
-                    if (at < p.cap) w.bucket[at] = RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)};
-                    ++at;
-                }
-            __syncthreads();
-            continue;
-        }
-        uint32_t pos = staged + off;
-#pragma unroll
-        for (int q = 0; q < kRadixPerThread; ++q)
-            if (r0 + q < hi && (c[q] >> kTop) == d1)
-                stage[pos++] = RadixEntry<C>{c[q], static_cast<uint32_t>(r0 + q)};
-        staged += tile_nb;
-        __syncthreads();
     }
-    if (staged) flush();
+    __syncwarp();
+    if (staged) wflush();
 }
 
 // After the last digit (prefix == X): from the bucket, entries with code > X join the

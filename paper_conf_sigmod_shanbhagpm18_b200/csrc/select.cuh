@@ -732,6 +732,10 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         take_bounds<Key, MIN>(st, cx, kth, publish);
         if (cnt > K) cnt = K;
     }
+    // every thread has read st (nflush, ties, limit) for this flush's decisions before
+    // thread 0 updates it (racecheck: without this barrier a late warp could read the
+    // incremented nflush and take a different `done` -- a divergent CSync)
+    CSync::sync();
     if (threadIdx.x == 0) {
         TOPK_STAT(0, 1ull);
         TOPK_STAT(1, static_cast<unsigned long long>(cnt0));
@@ -1256,13 +1260,15 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     for (uint32_t s = 0;; ++s) {
         const int slot = static_cast<int>(s % kStages);
         const uint32_t parity = (s / kStages) & 1u;
+        // warp-uniform wait (synccheck): a lane must not enter a collective while another
+        // lane of its warp is still polling the ring
         while (true) {
-            if (pending_req()) {
+            if (__any_sync(0xFFFFFFFFu, pending_req())) {
                 cbar_or(true);
                 collective();
                 continue;
             }
-            if (mbar_try_wait(&full[slot], parity)) break;
+            if (__all_sync(0xFFFFFFFFu, mbar_try_wait(&full[slot], parity))) break;
         }
         const uint32_t tile = st.tile[slot];
         if (tile == kEndTile) break;
