@@ -217,15 +217,23 @@ __device__ __forceinline__ void warp_append(RadixEntry<C>* list, uint32_t* cnt, 
 #define TOPK_RADIX_MATCH 0
 #endif
 constexpr int kHistNT = 256;
-constexpr size_t kHistSmem = size_t(kHistNT / 32) * kRadixBins * sizeof(uint32_t);  // 8 KB
+// kHistCopies histograms per warp (lane % kHistCopies), rows padded by one word so the
+// copies of one bin sit in different banks: U(0,1) floats put half the keys on one first
+// digit, and same-address shared atomics of a warp serialise
+#ifndef TOPK_HIST_COPIES
+#define TOPK_HIST_COPIES 1
+#endif
+constexpr int kHistCopies = TOPK_HIST_COPIES;
+constexpr int kHistRow = kRadixBins + 1;
 template <class Key, bool MIN, bool FIRST>
 __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
     using C = typename CodeOf<typename KeyTraits<Key>::E>::C;
-    __shared__ uint32_t hw[kHistNT / 32][kRadixBins];
+    constexpr int kRows = kHistNT / 32 * kHistCopies;
+    __shared__ uint32_t hw[kRows][kHistRow];
     const int warp = threadIdx.x >> 5;
     const RadixWs<C> w = radix_ws<C>(p.ws, p.G, p.k);
-    for (int i = threadIdx.x; i < (kHistNT / 32) * kRadixBins; i += kHistNT) (&hw[0][0])[i] = 0u;
-    uint32_t* mine = hw[warp];
+    for (int i = threadIdx.x; i < kRows * kHistRow; i += kHistNT) (&hw[0][0])[i] = 0u;
+    uint32_t* mine = hw[warp * kHistCopies + (threadIdx.x & 31) % kHistCopies];
     const C prefix = FIRST ? C(0) : w.st->prefix;
     const uint32_t shift = FIRST ? sizeof(C) * 8 - 8 : w.st->shift;
     const bool from_bucket = !FIRST && w.st->bucket_ok;
@@ -240,10 +248,16 @@ __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
         const Key* keys = static_cast<const Key*>(p.keys);
         const uint64_t lo = blockIdx.x * p.slice, hi = min(p.n, lo + p.slice);
         constexpr int kT = kHistNT * kRadixPerThread;
+        // two tiles in flight per thread (the loads of the next tile are issued before the
+        // counts of the current one: the pass is bound by memory-level parallelism)
+        C cn[kRadixPerThread];
+        load_codes<Key, MIN>(keys, hi, lo + threadIdx.x * kRadixPerThread, cn);
         for (uint64_t t0 = lo; t0 < hi; t0 += kT) {
             C c[kRadixPerThread];
+#pragma unroll
+            for (int q = 0; q < kRadixPerThread; ++q) c[q] = cn[q];
             const uint64_t r0 = t0 + threadIdx.x * kRadixPerThread;
-            load_codes<Key, MIN>(keys, hi, r0, c);
+            if (t0 + kT < hi) load_codes<Key, MIN>(keys, hi, r0 + kT, cn);
 #pragma unroll
             for (int q = 0; q < kRadixPerThread; ++q) {
                 const bool ok = r0 + q < hi && has_prefix(c[q], prefix, shift);
@@ -263,7 +277,7 @@ __global__ void __launch_bounds__(kHistNT) radix_hist(const RadixParams p) {
     for (int b = threadIdx.x; b < kRadixBins; b += kHistNT) {
         uint32_t s = 0;
 #pragma unroll
-        for (int wv = 0; wv < kHistNT / 32; ++wv) s += hw[wv][b];
+        for (int wv = 0; wv < kRows; ++wv) s += hw[wv][b];
         if (s) atomicAdd(&w.hist[b], s);  // the pass's total (radix_choose reads and zeroes it)
     }
 }
