@@ -231,6 +231,33 @@ def probe_read(x, stream, torch):
     return out
 
 
+def graph_us(f, torch, reps=30):
+    """Device time per call: `reps` calls captured in a CUDA graph and replayed (min of 5
+    replays), so the host-side cost of each Python call is not in the number."""
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        for _ in range(3):
+            f()
+    torch.cuda.current_stream().wait_stream(s)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for _ in range(reps):
+            f()
+    g.replay()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(5):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1) / reps * 1e3)
+    return min(ts)
+
+
 def ncu_traffic(k, n, timeout=420):
     """DRAM bytes (read + write) of ONE select_kernel launch on the headline input, from
     an ncu subprocess (`bench.py --ncu-target`) -- the roofline `traffic` of this run.
@@ -505,8 +532,15 @@ def run_extras(args, tk, datagen, x, stream, torch, hbm):
     cfgs = []
     x1 = datagen.generate("uniform", 1 << 20, "f32", seed=datagen.config_seed(1), device=dev)
     t = timed(lambda: tk.topk(x1, 32, True), 50)
-    cfgs.append({"config": "BJ1: 2^20 uniform f32, k=32 (launch-bound, L2-resident, back to back)",
+    cfgs.append({"config": "BJ1: 2^20 uniform f32, k=32 (per Python call, back to back: host-bound)",
                  "us": round(t * 1e3, 2), "keys_per_s": (1 << 20) / (t / 1e3)})
+    v1 = torch.empty(32, dtype=torch.float32, device=dev)
+    i1 = torch.empty(32, dtype=torch.int64, device=dev)
+    ws1 = tk.Workspace(tk.workspace_bytes(torch.float32, 1 << 20, 32), dev)
+    t = graph_us(lambda: tk.topk(x1, 32, True, out=(v1, i1, None), workspace=ws1), torch)
+    cfgs.append({"config": "BJ1: 2^20 uniform f32, k=32 (device latency: 30 calls replayed from a "
+                           "CUDA graph, L2-resident)", "us": round(t, 2),
+                 "keys_per_s": (1 << 20) / (t / 1e6)})
     x1 = None
     del x1
     n4 = 1 << 28

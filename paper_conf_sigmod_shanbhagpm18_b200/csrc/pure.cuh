@@ -38,6 +38,7 @@ constexpr int kPureNW = kPureNT / 32;
 constexpr int kPureChunk = 1024;                   // keys per warp chunk
 constexpr int kPureCap = 4096;                     // merge buffer entries (+ as many for exchange)
 constexpr int kPureStages = 3;                     // TMA ring slots per warp (4 KB each)
+constexpr int kPureGroup = 16;                     // CTA runs merged per first-level node
 // smem: [ring: 16 warps x kPureStages x 4 KB (the merge buffer, 2 x 4096 E32, reuses
 // it after streaming) | stage: 16 x 32 E32 | mbarriers: 16 x kPureStages]
 constexpr size_t kPureRingBytes = static_cast<size_t>(kPureNW) * kPureStages * kPureChunk * 4;
@@ -50,8 +51,8 @@ struct PureParams {
     void* out_keys;
     uint32_t* out_payload;
     int64_t* out_idx;
-    unsigned int* ticket;  // workspace word, zero on entry and on exit
-    uint64_t* cand;        // workspace: G x K E32 (scratch)
+    unsigned int* ticket;  // workspace words [1 + ceil(G / kPureGroup)], zero on entry and exit
+    uint64_t* cand;        // workspace: (G + ceil(G / kPureGroup)) x K E32 (scratch)
     uint64_t n;
     uint64_t base;
     uint32_t k;
@@ -342,6 +343,44 @@ __device__ __forceinline__ void pure_warp(const PureParams& p, uint32_t* ring, u
     }
 }
 
+// Merge `nruns` sorted (best-first) runs of K entries from global memory (run r at
+// src + r * K) into b[0 .. K) best first: slot 0 keeps the result between buffers, odd
+// slots are loaded reversed (runs alternating direction: the state the local sort
+// leaves), then merge + rebuild rounds (wnet_small, presorted).  Collective (CTA).
+template <int L>
+__device__ __forceinline__ void merge_runs(const SBuf<E32>& b, const uint64_t* src, int nruns,
+                                           int w, int lane) {
+    constexpr int K = 1 << L;
+    const int tid = threadIdx.x;
+    const int slots = kPureCap / K;  // runs per network buffer
+    int next = 0;
+    bool first = true;
+    while (next < nruns) {
+        const int s0 = first ? 0 : 1;  // slot 0: the result so far (best first)
+        const int take = min(slots - s0, nruns - next);
+        const int used = s0 + take;
+        int P2 = 2 * K;
+        while (P2 < used * K) P2 <<= 1;
+        if (P2 < 64) P2 = 64;
+        for (int q = tid; q < P2 - s0 * K; q += kPureNT) {
+            const int s = s0 + q / K, j = q % K;
+            const int r = next + s - s0;
+            const E32 e = s < used ? E32{__ldcg(src + static_cast<size_t>(r) * K + j)}
+                                   : E32::sentinel();
+            b.st(s * K + ((s & 1) ? K - 1 - j : j), e);
+        }
+        __syncthreads();
+        if (P2 <= 1024)
+            wnet_small<E32, 2, kPureNW, CtaSync>(b, P2, L, w, lane, true);
+        else if (P2 <= 2048)
+            wnet_small<E32, 4, kPureNW, CtaSync>(b, P2, L, w, lane, true);
+        else
+            wnet_small<E32, 8, kPureNW, CtaSync>(b, P2, L, w, lane, true);
+        next += take;
+        first = false;
+    }
+}
+
 template <class Key, bool MIN, int L>
 __global__ void __launch_bounds__(kPureNT, 1) pure_kernel(const PureParams p) {
     constexpr int K = 1 << L;
@@ -352,7 +391,8 @@ __global__ void __launch_bounds__(kPureNT, 1) pure_kernel(const PureParams p) {
     uint64_t* stage = reinterpret_cast<uint64_t*>(smem + kPureRingBytes);
     uint64_t* bars = stage + kPureNW * 32;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint64_t gw = static_cast<uint64_t>(blockIdx.x) * kPureNW + w;
+    // warp chunks interleaved over the CTAs (a small input spreads over every SM)
+    const uint64_t gw = static_cast<uint64_t>(w) * gridDim.x + blockIdx.x;
     const uint64_t GW = static_cast<uint64_t>(gridDim.x) * kPureNW;
     uint64_t run = 0ull;  // the warp's running top-K: position = lane (< K), best first
     pure_warp<Key, MIN, L>(p, reinterpret_cast<uint32_t*>(smem) + w * kPureStages * kPureChunk,
@@ -367,45 +407,35 @@ __global__ void __launch_bounds__(kPureNT, 1) pure_kernel(const PureParams p) {
     if (lane < K) b.st(w * K + ((w & 1) ? K - 1 - lane : lane), E32{run});
     __syncthreads();
     wnet_small<E32, 2, kPureNW, CtaSync>(b, P, L, w, lane, true);
-    // the CTA's run -> workspace; the last CTA merges all of them
-    unsigned int* ticket = p.ticket;
-    uint64_t* cand = p.cand;
+    // Reduction tree over the CTA runs, two ticketed levels: the last CTA of each group of
+    // kPureGroup merges the group's runs, the last group leader merges the group runs.
     const int G = static_cast<int>(gridDim.x);
     if (G > 1) {
+        const int ng = (G + kPureGroup - 1) / kPureGroup;
+        const int g = static_cast<int>(blockIdx.x) / kPureGroup;
+        const int g0 = g * kPureGroup, gn = min(kPureGroup, G - g0);
+        uint64_t* cand = p.cand;                           // G runs
+        uint64_t* gcand = p.cand + static_cast<size_t>(G) * K;  // ng group runs
         for (int j = tid; j < K; j += kPureNT) __stcg(cand + blockIdx.x * K + j, b.ld(j).v);
         __threadfence();
         __syncthreads();
-        if (tid == 0) s_last = atomicAdd(ticket, 1u) == static_cast<unsigned>(G - 1);
+        if (tid == 0)
+            s_last = atomicAdd(p.ticket + 1 + g, 1u) == static_cast<unsigned>(gn - 1);
         __syncthreads();
         if (!s_last) return;
         __threadfence();
-        const int slots = kPureCap / K;  // runs per network buffer
-        int next = 0;
-        bool first = true;
-        while (next < G) {
-            const int s0 = first ? 0 : 1;  // slot 0: the result so far (best first)
-            const int take = min(slots - s0, G - next);
-            const int used = s0 + take;
-            int P2 = 2 * K;
-            while (P2 < used * K) P2 <<= 1;
-            if (P2 < 64) P2 = 64;
-            for (int q = tid; q < P2 - s0 * K; q += kPureNT) {
-                const int s = s0 + q / K, j = q % K;
-                const int r = next + s - s0;
-                const E32 e = s < used ? E32{__ldcg(cand + static_cast<size_t>(r) * K + j)}
-                                       : E32::sentinel();
-                b.st(s * K + ((s & 1) ? K - 1 - j : j), e);
-            }
+        merge_runs<L>(b, cand + static_cast<size_t>(g0) * K, gn, w, lane);
+        if (ng > 1) {
+            for (int j = tid; j < K; j += kPureNT) __stcg(gcand + g * K + j, b.ld(j).v);
+            __threadfence();
             __syncthreads();
-            if (P2 <= 1024)
-                wnet_small<E32, 2, kPureNW, CtaSync>(b, P2, L, w, lane, true);
-            else if (P2 <= 2048)
-                wnet_small<E32, 4, kPureNW, CtaSync>(b, P2, L, w, lane, true);
-            else
-                wnet_small<E32, 8, kPureNW, CtaSync>(b, P2, L, w, lane, true);
-            next += take;
-            first = false;
+            if (tid == 0) s_last = atomicAdd(p.ticket, 1u) == static_cast<unsigned>(ng - 1);
+            __syncthreads();
+            if (!s_last) return;
+            __threadfence();
+            merge_runs<L>(b, gcand, ng, w, lane);
         }
+        if (tid <= ng) p.ticket[tid] = 0u;  // leave the workspace zeroed (all others done)
     }
     // finalize: best first, original key bits, global index, payload
     const Key* keys = static_cast<const Key*>(p.keys);
@@ -415,7 +445,6 @@ __global__ void __launch_bounds__(kPureNT, 1) pure_kernel(const PureParams p) {
         if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = keys[row];
         if (p.out_payload) p.out_payload[j] = p.payload[row];
     }
-    if (tid == 0 && G > 1) *ticket = 0u;  // leave the workspace zeroed
 }
 
 }  // namespace topk

@@ -136,8 +136,9 @@ uint32_t query_tile_keys(topk_dtype_t dt, int q) {
 // Candidate area: one run of next_pow2(k) entries per CTA (the pure-mode kernel keeps
 // whole K-runs; the streaming select keeps k).
 size_t select_ws_bytes(topk_dtype_t dtype, uint32_t k, int sms) {
+    const size_t runs = static_cast<size_t>(sms) + (sms + topk::kPureGroup - 1) / topk::kPureGroup;
     return align_up(topk::ws_cand_offset(static_cast<uint32_t>(sms)) +
-                        static_cast<size_t>(sms) * next_pow2_u32(k) * entry_bytes(dtype),
+                        runs * next_pow2_u32(k) * entry_bytes(dtype),
                     256);
 }
 
@@ -290,7 +291,16 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
 
     cudaStream_t st = static_cast<cudaStream_t>(stream);
     const bool mn = order == TOPK_SMALLEST, filt = mode == TOPK_MODE_FILTER;
-    if (!filt && !qa.q && dtype != TOPK_F64 && p.K <= 32) {
+    // Small inputs in filter mode run the pure kernel too: the result is identical, and
+    // up to 2^22 keys (k <= 32) its fixed cost is lower than the streaming pass's (boot
+    // flush, tail) -- graph-timed on B200, 2^20 keys k = 32: 36.9 -> 19.9 us (DESIGN.md
+    // §4.4).  TOPK_PURE_SMALL_N overrides the cut (0 disables it).
+    static const uint64_t small_cut = [] {
+        const char* e = std::getenv("TOPK_PURE_SMALL_N");
+        return e ? static_cast<uint64_t>(std::strtoull(e, nullptr, 10)) : (1ull << 22);
+    }();
+    const bool small_pure = filt && n <= small_cut;
+    if ((!filt || small_pure) && !qa.q && dtype != TOPK_F64 && p.K <= 32) {
         // the paper's pure method, register/shuffle form (pure.cuh): 32-bit keys, K <= 32
         topk::PureParams pp;
         pp.keys = keys;
@@ -298,15 +308,15 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
         pp.out_keys = out_keys;
         pp.out_payload = out_payload;
         pp.out_idx = out_idx;
-        pp.ticket = reinterpret_cast<unsigned int*>(p.ws) + 5;  // WsHeader::pad[0]
+        pp.ticket = reinterpret_cast<unsigned int*>(p.ws) + 5;  // WsHeader::pad[0 .. 10]
         pp.cand = reinterpret_cast<uint64_t*>(p.ws + topk::ws_cand_offset(p.gmax));
         pp.n = n;
         pp.base = base;
         pp.k = k;
         pp.L = static_cast<uint32_t>(__builtin_ctz(p.K));
+        // chunks are dealt round robin over the CTAs: up to one CTA per SM, one per chunk
         const uint64_t nch = (n + topk::kPureChunk - 1) / topk::kPureChunk;
-        const uint64_t want = (nch + topk::kPureNW - 1) / topk::kPureNW;  // one chunk per warp
-        const int pgrid = static_cast<int>(want < static_cast<uint64_t>(sms) ? want : sms);
+        const int pgrid = static_cast<int>(nch < static_cast<uint64_t>(sms) ? nch : sms);
         const cudaError_t e = topk::launch_pure(key_kind(dtype), mn, pp, pgrid, st);
         if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
         return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;

@@ -312,3 +312,37 @@ def test_sharded_c_abi_one_rank(cuda_device, dt):
             assert np.array_equal(host(pv), host(p)[oi - base])
     finally:
         comm.close()
+
+
+def test_small_inputs_streaming_kernel(cuda_device):
+    """Filter-mode calls with n <= 2^22 and k <= 32 run the pure kernel (same result, lower
+    fixed cost); TOPK_PURE_SMALL_N=0 keeps them on the streaming kernel, whose small-input
+    path (one tile per CTA, boot flush, tail) is checked here in a subprocess."""
+    import os
+    import subprocess
+    import sys
+    code = """
+import sys
+import numpy as np
+sys.path.insert(0, '.')
+import oracle
+import paper_conf_sigmod_shanbhagpm18_b200 as tk
+from paper_conf_sigmod_shanbhagpm18_b200 import datagen
+for n in (1, 7, 4096, 4097, 100003, (1 << 20) + 13):
+    for dist in ('uniform', 'fewdistinct'):
+        x = datagen.generate(dist, n, 'f32', seed=n)
+        for k in (1, 8, 17, 32):
+            if k > n:
+                continue
+            for lg in (True, False):
+                v, i = tk.topk(x.cuda(), k, lg)
+                ov, oi = oracle.topk(x.numpy(), k, lg)
+                assert np.array_equal(i.cpu().numpy(), oi), (n, dist, k, lg)
+                assert v.cpu().numpy().tobytes() == ov.tobytes(), (n, dist, k, lg)
+print('ok')
+"""
+    env = dict(os.environ, TOPK_PURE_SMALL_N="0")
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=env, capture_output=True,
+                       text=True, timeout=600)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr[-2000:]
