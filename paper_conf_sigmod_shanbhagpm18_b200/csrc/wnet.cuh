@@ -123,12 +123,21 @@ __device__ __forceinline__ void wrebuild(E (&x)[R], int lane, uint32_t e0, int L
     for (int b = L - 1; b >= 0; --b) wstep<E, R>(x, lane, e0, b, L);
 }
 
-// Register pass over 512-entry chunks of b[0..P): steps b = hi .. 0 with direction
-// bit d (all within a chunk: bits 0-3 registers, 4-8 shuffles).
+// Entries per lane of a phase-A chunk: 16 (a 512-entry chunk) for 8-byte entries; 8 (256)
+// for the 12/16-byte entries of 64-bit codes and compound keys -- 16 of those would take
+// 48-64 registers per thread and spill under the kernel's 128-register cap.
+template <class E>
+struct WChunk {
+    static constexpr int R = sizeof(E) > 8 ? 8 : 16;
+    static constexpr int B = sizeof(E) > 8 ? 8 : 9;  // element bits inside a chunk
+};
+
+// Register pass over 32 R-entry chunks of b[0..P): steps b = hi .. 0 with direction
+// bit d (all within a chunk: low bits registers, the next 5 shuffles).
 template <class E, int NW>
 __device__ __forceinline__ void wchunk_steps(const SBuf<E>& b, int P, int hi, int d, int w,
                                              int lane) {
-    constexpr int RA = 16;
+    constexpr int RA = WChunk<E>::R;
 #pragma unroll 1
     for (int base = w * 32 * RA; base < P; base += NW * 32 * RA) {
         E x[RA];
@@ -172,14 +181,15 @@ __device__ __forceinline__ void wsmem_step(const SBuf<E>& b, int P, int bb, int 
 // 0-8 run in registers / shuffles; the rare steps on bits 9-10 (K >= 1024) in shared memory.
 template <class E, int NW, class Sync>
 __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
-    constexpr int RA = 16;  // phase A: 512 entries per warp chunk
-    constexpr int RB = 8;   // phase B: 256 outputs per warp per round
+    constexpr int RA = WChunk<E>::R;  // phase A: 32 RA entries per warp chunk
+    constexpr int CB = WChunk<E>::B;  // log2 of that
+    constexpr int RB = 8;             // phase B: 256 outputs per warp per round
     static_assert(NW * 32 * RB >= 2048, "phase B: one chunk of 256 outputs per warp");
     const int K = 1 << L;
-    // Phase A -- local sort into min(K, 512)-runs in registers.  Small buffers use
+    // Phase A -- local sort into min(K, 2^CB)-runs in registers.  Small buffers use
     // 256-entry chunks (8 per lane) so twice as many warps share the latency-bound
-    // step chain; K >= 512 or P > 2048 use 512-entry chunks (16 per lane).
-    const int LA = L < 9 ? L : 9;
+    // step chain; otherwise 32 RA-entry chunks.
+    const int LA = L < CB ? L : CB;
     if (L <= 8 && P <= 8 * 256 && NW >= 8) {
         constexpr int R8 = 8;
         const int base = w * 32 * R8;
@@ -221,15 +231,15 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
         }
     }
     Sync::sync();
-    // local-sort stages beyond 512-runs (len 512, 1024): bits >= 9 in smem, 8..0 in registers
+    // local-sort stages beyond chunk-size runs: bits >= CB in smem, CB-1 .. 0 in registers
 #pragma unroll 1
-    for (int d = 10; d <= L; ++d) {
+    for (int d = CB + 1; d <= L; ++d) {
 #pragma unroll 1
-        for (int bb = d - 1; bb >= 9; --bb) wsmem_step<E, NW * 32, Sync>(b, P, bb, d);
-        wchunk_steps<E, NW>(b, P, 8, d, w, lane);
+        for (int bb = d - 1; bb >= CB; --bb) wsmem_step<E, NW * 32, Sync>(b, P, bb, d);
+        wchunk_steps<E, NW>(b, P, CB - 1, d, w, lane);
         Sync::sync();
     }
-    if (L >= 9) {
+    if (L >= CB) {
         // Phase B for K >= 512: merge through registers + shared memory, rebuild with
         // the same hybrid steps.
 #pragma unroll 1
@@ -255,8 +265,8 @@ __device__ void wnet_topk(const SBuf<E>& b, int P, int L, int w, int lane) {
             Sync::sync();
             P = half;
 #pragma unroll 1
-            for (int bb = L - 1; bb >= 9; --bb) wsmem_step<E, NW * 32, Sync>(b, P, bb, L);
-            wchunk_steps<E, NW>(b, P, 8, L, w, lane);
+            for (int bb = L - 1; bb >= CB; --bb) wsmem_step<E, NW * 32, Sync>(b, P, bb, L);
+            wchunk_steps<E, NW>(b, P, CB - 1, L, w, lane);
             Sync::sync();
         }
         return;
