@@ -47,6 +47,12 @@ namespace topk {
 #ifndef TOPK_STAGES
 #define TOPK_STAGES 5
 #endif
+#ifndef TOPK_FINAL_CODE_MIN
+#define TOPK_FINAL_CODE_MIN 1025  // measured: k = 256 365.2 -> 362.5 us, increasing 366 -> 359 us
+#endif
+#ifndef TOPK_TAIL_ROWS
+#define TOPK_TAIL_ROWS 3
+#endif
 #ifndef TOPK_LIMIT2
 #define TOPK_LIMIT2 1024  // bag limit between the boot flush and the second flush
 #endif
@@ -681,7 +687,10 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
     bool done = false;
     // (tie-heavy input -- a code bound cannot separate equal codes -- makes the code
     // path useless: after it failed once, stream flushes go straight to the exact path)
-    const bool try_code = !st->ties && (publish || (cnt > 2 * K && K <= (1 << cx.Lp)));
+    // (a final flush of a bag the small exact network can take directly skips the code
+    // network: TOPK_FINAL_CODE_MIN is the smallest such bag that still goes through it)
+    const bool try_code = !st->ties && (publish || (cnt > 2 * K && K <= (1 << cx.Lp) &&
+                                                    cnt >= TOPK_FINAL_CODE_MIN));
     bool tried = false;
     if (cx.filter && cx.Lp >= 0 && !(c_dbg & 1) && try_code) {
         tried = true;
@@ -1332,6 +1341,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // (1) Rank bound over the final runs (tail form of the flush bound): row j holds
         // each run's 2^j-th best; the t-th largest (t = ceil(k / 2^j) <= G) bounds the
         // global k-th best.  All loads in one parallel pass.
+        if (cx.nrows > TOPK_TAIL_ROWS) cx.nrows = TOPK_TAIL_ROWS;
         for (int q = tid; q < cx.nrows * cx.G; q += kNC) {
             const int ji = cx.j_lo + q / cx.G, cc = q % cx.G;
             scratch[q] = bound_word(cand.ld(static_cast<size_t>(cc) * k + (1u << ji) - 1u));
