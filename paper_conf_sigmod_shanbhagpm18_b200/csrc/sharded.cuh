@@ -54,7 +54,7 @@ NcclApi& nccl_api() {
 }
 
 struct ShardLayout {
-    size_t sel, lk, li, lp, gk, gi, gp, total;
+    size_t sel, lk, li, lp, lr, gk, gi, gp, gr, total;
 };
 
 ShardLayout shard_layout(topk_dtype_t dtype, uint64_t n_local, uint32_t k, int nranks) {
@@ -65,10 +65,12 @@ ShardLayout shard_layout(topk_dtype_t dtype, uint64_t n_local, uint32_t k, int n
     L.lk = align_up(sel_bytes, 256);
     L.li = L.lk + align_up(static_cast<size_t>(k) * ks, 256);
     L.lp = L.li + align_up(static_cast<size_t>(k) * 8, 256);
-    L.gk = L.lp + align_up(static_cast<size_t>(k) * 4, 256);
+    L.lr = L.lp + align_up(static_cast<size_t>(k) * 4, 256);
+    L.gk = L.lr + 256;
     L.gi = L.gk + align_up(static_cast<size_t>(nranks) * k * ks, 256);
     L.gp = L.gi + align_up(static_cast<size_t>(nranks) * k * 8, 256);
-    L.total = L.gp + align_up(static_cast<size_t>(nranks) * k * 4, 256);
+    L.gr = L.gp + align_up(static_cast<size_t>(nranks) * k * 4, 256);
+    L.total = L.gr + align_up(static_cast<size_t>(nranks) * 16, 256);
     return L;
 }
 
@@ -135,20 +137,26 @@ topk_status_t topk_select_sharded(topk_dtype_t dtype, const void* keys, const ui
                                   w + L.lk, payload ? reinterpret_cast<uint32_t*>(w + L.lp) : nullptr,
                                   reinterpret_cast<int64_t*>(w + L.li), w + L.sel, L.lk, stream);
     if (s != TOPK_OK) return s;
-    // (2) all-gather the candidates of every rank
+    // (2) all-gather the candidates of every rank, and every rank's row range (the merge
+    // narrows its entries when the ranges increase rank by rank)
     cudaStream_t st = static_cast<cudaStream_t>(stream);
+    const uint64_t range[2] = {base, n_local};  // pageable: staged at once, stream-ordered
+    if (cudaMemcpyAsync(w + L.lr, range, sizeof(range), cudaMemcpyHostToDevice, st) != cudaSuccess)
+        return TOPK_ERR_CUDA;
     ncclComm_t c = static_cast<ncclComm_t>(comm);
     if (a.group_start() != ncclSuccess) return TOPK_ERR_NCCL;
     ncclResult_t r = a.all_gather(w + L.lk, w + L.gk, k * ks, ncclUint8, c, st);
     if (r == ncclSuccess) r = a.all_gather(w + L.li, w + L.gi, k, ncclInt64, c, st);
     if (r == ncclSuccess && payload) r = a.all_gather(w + L.lp, w + L.gp, k, ncclUint32, c, st);
+    if (r == ncclSuccess) r = a.all_gather(w + L.lr, w + L.gr, 2, ncclUint64, c, st);
     const ncclResult_t r2 = a.group_end();
     if (r != ncclSuccess || r2 != ncclSuccess) return TOPK_ERR_NCCL;
     // (3) the global step: exact top-k of the G sorted candidate runs
     return merge_total(dtype, w + L.gk, reinterpret_cast<const int64_t*>(w + L.gi),
                        payload ? reinterpret_cast<const uint32_t*>(w + L.gp) : nullptr,
                        static_cast<uint64_t>(nranks) * k, k, true, k, order, out_keys,
-                       out_payload, out_idx, stream);
+                       out_payload, out_idx, stream, false,
+                       reinterpret_cast<const uint64_t*>(w + L.gr));
 }
 
 topk_status_t topk_f32_sharded(const float* keys, uint64_t n_local, uint64_t base, uint32_t k,

@@ -151,7 +151,8 @@ static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
                                  const int64_t* cand_idx, const uint32_t* cand_payload,
                                  uint64_t total, uint32_t run_len, bool sorted, uint32_t k,
                                  topk_order_t order, void* out_keys, uint32_t* out_payload,
-                                 int64_t* out_idx, void* stream);
+                                 int64_t* out_idx, void* stream, bool ordered = false,
+                                 const uint64_t* ranges = nullptr);
 // chunked-input helpers (used by topk_workspace_bytes / topk_select).  Chunk length
 // 2^31 keys; TOPK_CHUNK_N (multiple of 4) overrides it so tests can exercise the
 // chunked path on small inputs.
@@ -377,9 +378,10 @@ topk_status_t topk_select(topk_dtype_t dtype, const void* keys, const uint32_t* 
         total += kc;
     }
     // the chunks' results are sorted runs of k entries (the last one may be shorter)
+    // chunks in order: chunk c's ids all below chunk c+1's
     return merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
                        payload ? reinterpret_cast<const uint32_t*>(w + L.cp) : nullptr, total, k,
-                       true, k, order, out_keys, out_payload, out_idx, stream);
+                       true, k, order, out_keys, out_payload, out_idx, stream, true);
 }
 
 topk_status_t topk_query(topk_dtype_t dtype, const void* keys, const float* rank_b,
@@ -773,7 +775,7 @@ topk_status_t topk_select_host(topk_dtype_t dtype, const void* h_keys, uint64_t 
     }
     topk_status_t r = merge_total(dtype, w + L.ck, reinterpret_cast<const int64_t*>(w + L.ci),
                                   nullptr, total, k, true, k, order, w + L.ok, nullptr,
-                                  reinterpret_cast<int64_t*>(w + L.oi), stream);
+                                  reinterpret_cast<int64_t*>(w + L.oi), stream, true);
     if (r != TOPK_OK) return r;
     if (h_out_keys &&
         cudaMemcpyAsync(h_out_keys, w + L.ok, k * ks, cudaMemcpyDeviceToHost, st) != cudaSuccess)
@@ -806,7 +808,8 @@ static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
                                  const int64_t* cand_idx, const uint32_t* cand_payload,
                                  uint64_t total, uint32_t run_len, bool sorted, uint32_t k,
                                  topk_order_t order, void* out_keys, uint32_t* out_payload,
-                                 int64_t* out_idx, void* stream) {
+                                 int64_t* out_idx, void* stream, bool ordered,
+                                 const uint64_t* ranges) {
     if (!valid_dtype(dtype) || !valid_order(order)) return TOPK_ERR_INVALID_ARG;
     if (!cand_keys || !cand_idx || total == 0) return TOPK_ERR_INVALID_ARG;
     if (total > 65536 || k == 0 || k > TOPK_MAX_K || k > total) return TOPK_ERR_INVALID_ARG;
@@ -824,6 +827,8 @@ static topk_status_t merge_total(topk_dtype_t dtype, const void* cand_keys,
     p.total = static_cast<uint32_t>(total);
     p.run_len = run_len == 0 ? 1u : run_len;
     p.sorted = sorted ? 1u : 0u;
+    p.ordered = sorted ? (ordered ? 1u : (ranges ? 0u : 2u)) : 0u;
+    p.ranges = sorted ? ranges : nullptr;
     p.k = k;
     p.K = next_pow2_u32(k);
     cudaStream_t st = static_cast<cudaStream_t>(stream);

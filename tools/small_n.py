@@ -32,14 +32,15 @@ def graph_us(f, reps=30):
     return round(min(ts), 2)
 
 
-for lg in (12, 16, 18, 20, 22, 24, 26):
-    n = 1 << lg
-    x = datagen.generate("uniform", n, "f32", seed=5, device="cuda")
-    for k in (8, 32):
-        row = {"log2n": lg, "k": k}
-        v = torch.empty(k, dtype=torch.float32, device="cuda")
-        i = torch.empty(k, dtype=torch.int64, device="cuda")
-        ws = tk.Workspace(tk.workspace_bytes(torch.float32, n, k), "cuda")
-        for mode in ("filter", "pure"):
-            row[mode] = graph_us(lambda: tk.topk(x, k, mode=mode, out=(v, i, None), workspace=ws))
-        print(json.dumps(row), flush=True)
+if __name__ == "__main__":
+    for lg in (12, 16, 18, 20, 22, 24, 26):
+        n = 1 << lg
+        x = datagen.generate("uniform", n, "f32", seed=5, device="cuda")
+        for k in (8, 32):
+            row = {"log2n": lg, "k": k}
+            v = torch.empty(k, dtype=torch.float32, device="cuda")
+            i = torch.empty(k, dtype=torch.int64, device="cuda")
+            ws = tk.Workspace(tk.workspace_bytes(torch.float32, n, k), "cuda")
+            for mode in ("filter", "pure"):
+                row[mode] = graph_us(lambda: tk.topk(x, k, mode=mode, out=(v, i, None), workspace=ws))
+            print(json.dumps(row), flush=True)
