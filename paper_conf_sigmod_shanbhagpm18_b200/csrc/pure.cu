@@ -1,5 +1,5 @@
 // pure.cu -- instantiations and launcher of the pure-mode kernel (pure.cuh): 32-bit keys,
-// max / min order, K = 2^L for L = 0 .. 5.
+// max / min order, K = 2^L for L = 0 .. 5 (keys-only network) and 6 .. 8 (entries).
 #include <cuda_runtime.h>
 
 #include "dispatch.h"
@@ -18,6 +18,16 @@ cudaError_t launch_pure_l(const PureParams& p, int grid, cudaStream_t st) {
     return cudaGetLastError();
 }
 
+template <class Key, bool MIN, int L>
+cudaError_t launch_pure64_l(const PureParams& p, int grid, cudaStream_t st) {
+    static std::atomic<uint64_t> attr{0};  // per device (dispatch.h)
+    const cudaError_t e =
+        smem_attr_once(pure64_kernel<Key, MIN, L>, static_cast<int>(kPureSmem), attr);
+    if (e != cudaSuccess) return e;
+    pure64_kernel<Key, MIN, L><<<grid, kPureNT, kPureSmem, st>>>(p);
+    return cudaGetLastError();
+}
+
 template <class Key, bool MIN>
 cudaError_t launch_pure_k(const PureParams& p, int grid, cudaStream_t st) {
     switch (p.L) {
@@ -27,6 +37,9 @@ cudaError_t launch_pure_k(const PureParams& p, int grid, cudaStream_t st) {
         case 3: return launch_pure_l<Key, MIN, 3>(p, grid, st);
         case 4: return launch_pure_l<Key, MIN, 4>(p, grid, st);
         case 5: return launch_pure_l<Key, MIN, 5>(p, grid, st);
+        case 6: return launch_pure64_l<Key, MIN, 6>(p, grid, st);
+        case 7: return launch_pure64_l<Key, MIN, 7>(p, grid, st);
+        case 8: return launch_pure64_l<Key, MIN, 8>(p, grid, st);
     }
     return cudaErrorInvalidValue;
 }

@@ -447,4 +447,160 @@ __global__ void __launch_bounds__(kPureNT, 1) pure_kernel(const PureParams p) {
     }
 }
 
+// ---- K = 64 .. 256: (code, index) entries through the network -------------------------
+// A run of K no longer fits the keys-only fold layout with a cheap recovery (K entries of
+// every 1024-key chunk would need sorting), so these K carry E32 = code << 32 | ~index
+// through every compare-exchange: per 512-key half chunk, 16 entries per lane (position
+// lane * 16 + r; key r * 32 + lane of the half, so the shared-memory reads are conflict-
+// free), local sort (Alg. 2) into K-runs and merge + rebuild rounds down to one run of K
+// (wnet.cuh register / shuffle steps), then merge + rebuild into the warp's running run
+// (same layout: positions 0 .. K - 1 in lanes 0 .. K / 16 - 1).
+
+template <class Key, bool MIN, int L>
+__device__ __forceinline__ void pure_warp64(const PureParams& p, uint32_t* ring, uint64_t* bars,
+                                            E32 (&run)[16], int lane, uint64_t gw, uint64_t GW) {
+    using KT = KeyTraits<Key>;
+    constexpr int K = 1 << L;
+    constexpr int RL = K / 16;  // lanes holding a run
+    static_assert(L >= 6 && L <= 8, "pure_warp64: K = 64 .. 256");
+    const Key* keys = static_cast<const Key*>(p.keys);
+    const uint64_t nch = (p.n + kPureChunk - 1) / kPureChunk;
+    const bool tma = (reinterpret_cast<uintptr_t>(keys) & 15u) == 0;
+    const uint64_t nfull = tma ? p.n / kPureChunk : 0;
+    const uint64_t policy = l2_evict_first_policy();
+    const uint32_t e0 = static_cast<uint32_t>(lane * 16);
+    if (lane == 0) {
+        for (int s = 0; s < kPureStages; ++s) mbar_init(&bars[s], 1);
+        fence_mbar_init();
+        for (int s = 0; s < kPureStages; ++s) {
+            const uint64_t ch = gw + s * GW;
+            if (ch < nfull) {
+                mbar_arrive_expect_tx(&bars[s], kPureChunk * 4);
+                tma_load_1d(ring + s * kPureChunk, keys + ch * kPureChunk, kPureChunk * 4,
+                            &bars[s], policy);
+            }
+        }
+    }
+    __syncwarp();
+    uint32_t it = 0;
+#pragma unroll 1
+    for (uint64_t ch = gw; ch < nch; ch += GW, ++it) {
+        const uint64_t c0 = ch * kPureChunk;
+        const bool full = ch < nfull;
+        const int slot = static_cast<int>(it % kPureStages);
+        if (full) mbar_wait(&bars[slot], (it / kPureStages) & 1u);
+        const Key* sk = reinterpret_cast<const Key*>(ring + slot * kPureChunk);
+#pragma unroll 1
+        for (int half = 0; half < 2; ++half) {
+            E32 x[16];
+#pragma unroll
+            for (int r = 0; r < 16; ++r) {
+                const uint32_t ci = static_cast<uint32_t>(half * 512 + r * 32 + lane);
+                const uint64_t i = c0 + ci;
+                const Key v = full ? sk[ci] : (i < p.n ? keys[i] : Key{});
+                x[r] = i < p.n ? E32::make(KT::template code<MIN>(v), static_cast<uint32_t>(i))
+                               : E32::sentinel();
+            }
+            if (full && half == 1) {  // the slot is consumed: prefetch the chunk after next
+                __syncwarp();
+                const uint64_t nx = ch + kPureStages * GW;
+                if (lane == 0 && nx < nfull) {
+                    mbar_arrive_expect_tx(&bars[slot], kPureChunk * 4);
+                    tma_load_1d(ring + slot * kPureChunk, keys + nx * kPureChunk, kPureChunk * 4,
+                                &bars[slot], policy);
+                }
+            }
+            // local sort (Alg. 2) into K-runs, then merge + rebuild (Alg. 4) rounds
+            // to one best-first run of K in positions 0 .. K - 1
+            wsort_runs<E32, 16>(x, lane, e0, L);
+#pragma unroll 1
+            for (int sb = L; sb < 9; ++sb) {
+                wstep<E32, 16>(x, lane, e0, sb, 9);  // merge: the lower keeps the better
+#pragma unroll 1
+                for (int b = L - 1; b >= 0; --b) wstep<E32, 16>(x, lane, e0, b, sb + 1);
+            }
+            // merge into the running run: run[j] vs chunk[K - 1 - j] (the chunk's run read
+            // backwards: lane RL - 1 - l, register 15 - r), then rebuild best first
+#pragma unroll
+            for (int r = 0; r < 16; ++r) {
+                const E32 y = shfl_xor_e(x[15 - r], RL - 1);
+                run[r] = lane < RL ? esel(better(run[r], y), run[r], y) : E32::sentinel();
+            }
+#pragma unroll 1
+            for (int b = L - 1; b >= 0; --b) wstep<E32, 16>(run, lane, e0, b, 9);
+        }
+    }
+}
+
+template <class Key, bool MIN, int L>
+__global__ void __launch_bounds__(kPureNT, 1) pure64_kernel(const PureParams p) {
+    constexpr int K = 1 << L;
+    constexpr int RL = K / 16;
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ int s_last;
+    SBuf<E32> b;
+    b.init(smem, 2 * kPureCap);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + kPureRingBytes) + kPureNW * 32;
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+    const uint64_t gw = static_cast<uint64_t>(w) * gridDim.x + blockIdx.x;
+    const uint64_t GW = static_cast<uint64_t>(gridDim.x) * kPureNW;
+    E32 run[16];
+#pragma unroll
+    for (int r = 0; r < 16; ++r) run[r] = E32::sentinel();
+    pure_warp64<Key, MIN, L>(p, reinterpret_cast<uint32_t*>(smem) + w * kPureStages * kPureChunk,
+                             bars + w * kPureStages, run, lane, gw, GW);
+    __syncthreads();  // the merge buffer reuses the rings
+    // CTA: the 16 warp runs (odd ones reversed), merge + rebuild rounds (wnet_small)
+    if (lane < RL) {
+#pragma unroll
+        for (int r = 0; r < 16; ++r) {
+            const int j = lane * 16 + r;
+            b.st(w * K + ((w & 1) ? K - 1 - j : j), run[r]);
+        }
+    }
+    __syncthreads();
+    constexpr int P = kPureNW * K;  // 1024 .. 4096
+    if constexpr (P <= 1024)
+        wnet_small<E32, 2, kPureNW, CtaSync>(b, P, L, w, lane, true);
+    else if constexpr (P <= 2048)
+        wnet_small<E32, 4, kPureNW, CtaSync>(b, P, L, w, lane, true);
+    else
+        wnet_small<E32, 8, kPureNW, CtaSync>(b, P, L, w, lane, true);
+    const int G = static_cast<int>(gridDim.x);
+    if (G > 1) {
+        const int ng = (G + kPureGroup - 1) / kPureGroup;
+        const int g = static_cast<int>(blockIdx.x) / kPureGroup;
+        const int g0 = g * kPureGroup, gn = min(kPureGroup, G - g0);
+        uint64_t* cand = p.cand;
+        uint64_t* gcand = p.cand + static_cast<size_t>(G) * K;
+        for (int j = tid; j < K; j += kPureNT) __stcg(cand + blockIdx.x * K + j, b.ld(j).v);
+        __threadfence();
+        __syncthreads();
+        if (tid == 0)
+            s_last = atomicAdd(p.ticket + 1 + g, 1u) == static_cast<unsigned>(gn - 1);
+        __syncthreads();
+        if (!s_last) return;
+        __threadfence();
+        merge_runs<L>(b, cand + static_cast<size_t>(g0) * K, gn, w, lane);
+        if (ng > 1) {
+            for (int j = tid; j < K; j += kPureNT) __stcg(gcand + g * K + j, b.ld(j).v);
+            __threadfence();
+            __syncthreads();
+            if (tid == 0) s_last = atomicAdd(p.ticket, 1u) == static_cast<unsigned>(ng - 1);
+            __syncthreads();
+            if (!s_last) return;
+            __threadfence();
+            merge_runs<L>(b, gcand, ng, w, lane);
+        }
+        if (tid <= ng) p.ticket[tid] = 0u;
+    }
+    const Key* keys = static_cast<const Key*>(p.keys);
+    for (int j = tid; j < static_cast<int>(p.k); j += kPureNT) {
+        const uint32_t row = b.ld(j).lidx();
+        if (p.out_idx) p.out_idx[j] = static_cast<int64_t>(p.base + row);
+        if (p.out_keys) static_cast<Key*>(p.out_keys)[j] = keys[row];
+        if (p.out_payload) p.out_payload[j] = p.payload[row];
+    }
+}
+
 }  // namespace topk

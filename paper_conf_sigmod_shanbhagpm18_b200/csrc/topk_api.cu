@@ -301,8 +301,8 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
         return e ? static_cast<uint64_t>(std::strtoull(e, nullptr, 10)) : (1ull << 22);
     }();
     const bool small_pure = filt && n <= small_cut;
-    if ((!filt || small_pure) && !qa.q && dtype != TOPK_F64 && p.K <= 32) {
-        // the paper's pure method, register/shuffle form (pure.cuh): 32-bit keys, K <= 32
+    if (((!filt && p.K <= 256) || (small_pure && p.K <= 32)) && !qa.q && dtype != TOPK_F64) {
+        // the paper's pure method, register/shuffle form (pure.cuh): 32-bit keys, K <= 256
         topk::PureParams pp;
         pp.keys = keys;
         pp.payload = payload;

@@ -83,3 +83,16 @@ def test_pure_special_values(cuda_device):
     for k in (1, 4, 32):
         check(x, k, True)
         check(x, k, False)
+
+
+@pytest.mark.parametrize("k", [33, 64, 100, 128, 129, 200, 256])
+def test_pure_entry_network(cuda_device, k):
+    """32 < k <= 256: the (code, index) entry network (pure64_kernel)."""
+    for n, dist in (((1 << 20) + 333, "uniform"), ((1 << 19) + 5, "fewdistinct"),
+                    (4097, "uniform"), ((1 << 21) + 1, "decreasing")):
+        x = datagen.generate(dist, n, "f32", seed=n + k)
+        check(x, k, True)
+        check(x, k, False)
+    xu = datagen.generate("uniform", (1 << 20) + 7, "u32", seed=k)
+    p = datagen.payload((1 << 20) + 7, seed=k)
+    check(xu, k, True, payload=p, base=77)
