@@ -17,8 +17,8 @@ import sys
 from collections import defaultdict
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-OUT = os.path.join(ROOT, "gpurun_out")
-PROF = os.path.join(ROOT, "profiles")
+OUT = os.environ.get("PROF_IN", os.path.join(ROOT, "gpurun_out"))
+PROF = os.environ.get("PROF_OUT", os.path.join(ROOT, "profiles"))
 
 KEYS = [
     "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
@@ -71,7 +71,7 @@ def to_bytes(v, unit):
 
 def main(rnd):
     os.makedirs(PROF, exist_ok=True)
-    traffic_path = os.path.join(PROF, "traffic.json")
+    traffic_path = os.path.join(PROF, "traffic_summary.json")  # (bench.py measures its own)
     traffic = json.load(open(traffic_path)) if os.path.exists(traffic_path) else {}
     for rep in sorted(glob.glob(os.path.join(OUT, f"prof_select_k*_{rnd}.ncu-rep"))):
         k = re.search(r"_k(\d+)_", rep).group(1)
