@@ -110,6 +110,15 @@ def workload(k, world=1, n_total=None):
             f"values+indices (BJ configs[4], strong scaling)")
 
 
+def shard_plan(rank, world, n_total=None):
+    """The rows rank `rank` of `world` owns: weak scaling (n_total None) -- 2^29 per rank,
+    global input world * 2^29; strong scaling -- n_total split into contiguous shards.
+    Returns (n_total, lo, hi): global rows [lo, hi)."""
+    if n_total is None:
+        n_total = world * N_PER_GPU
+    return n_total, n_total * rank // world, n_total * (rank + 1) // world
+
+
 def dist_env():
     r = int(os.environ.get("RANK", "0"))
     w = int(os.environ.get("WORLD_SIZE", "1"))
@@ -359,8 +368,7 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
     strong = args.n_total is not None
-    n_total = args.n_total if strong else world * N_PER_GPU
-    lo, hi = n_total * rank // world, n_total * (rank + 1) // world
+    n_total, lo, hi = shard_plan(rank, world, args.n_total)
     n = hi - lo  # this rank's shard: global rows [lo, hi)
     k = args.k
     stream = torch.cuda.current_stream(dev)
