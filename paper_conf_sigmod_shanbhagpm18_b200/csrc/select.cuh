@@ -50,6 +50,9 @@ namespace topk {
 #ifndef TOPK_FINAL_CODE_MIN
 #define TOPK_FINAL_CODE_MIN 1025  // measured: k = 256 365.2 -> 362.5 us, increasing 366 -> 359 us
 #endif
+#ifndef TOPK_FLUSH_ROWS
+#define TOPK_FLUSH_ROWS 2  // A/B: 3 -> 2 rows: k=256 362.5 -> 360.5 us, few-distinct 399 -> 394 (1 row: ties 1.5x slower)
+#endif
 #ifndef TOPK_TAIL_ROWS
 #define TOPK_TAIL_ROWS 3
 #endif
@@ -592,9 +595,12 @@ __device__ void take_bounds(CtaState<typename KeyTraits<Key>::E, Key>* st, const
             }
             CSync::sync();
         }
-        load_pub(cx);
+        // stream flushes rank TOPK_FLUSH_ROWS sample rows (the tail ranks all nrows)
+        Ctx cr = cx;
+        if (cr.nrows > TOPK_FLUSH_ROWS) cr.nrows = TOPK_FLUSH_ROWS;
+        load_pub(cr);
         CSync::sync();
-        rank_rows(st, cx);
+        rank_rows(st, cr);
     }
     if (threadIdx.x == 0) {
         if (!publish)

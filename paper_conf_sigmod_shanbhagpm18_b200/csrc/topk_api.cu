@@ -317,7 +317,13 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
         pp.L = static_cast<uint32_t>(__builtin_ctz(p.K));
         // chunks are dealt round robin over the CTAs: up to one CTA per SM, one per chunk
         const uint64_t nch = (n + topk::kPureChunk - 1) / topk::kPureChunk;
-        const int pgrid = static_cast<int>(nch < static_cast<uint64_t>(sms) ? nch : sms);
+        static const uint64_t grid_cap = [] {  // dev knob: TOPK_PURE_GRID (max CTAs)
+            const char* e = std::getenv("TOPK_PURE_GRID");
+            return e ? static_cast<uint64_t>(std::strtoull(e, nullptr, 10)) : 0ull;
+        }();
+        uint64_t cap = static_cast<uint64_t>(sms);
+        if (grid_cap > 0 && grid_cap < cap) cap = grid_cap;
+        const int pgrid = static_cast<int>(nch < cap ? nch : cap);
         const cudaError_t e = topk::launch_pure(key_kind(dtype), mn, pp, pgrid, st);
         if (e == cudaSuccess) g_launches.fetch_add(1, std::memory_order_relaxed);
         return e == cudaSuccess ? TOPK_OK : TOPK_ERR_CUDA;
