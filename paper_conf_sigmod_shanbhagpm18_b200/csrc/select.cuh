@@ -50,6 +50,16 @@ namespace topk {
 #ifndef TOPK_FINAL_CODE_MIN
 #define TOPK_FINAL_CODE_MIN 1025  // measured: k = 256 365.2 -> 362.5 us, increasing 366 -> 359 us
 #endif
+// Rows per consumer thread of a query-form stage (one TMA slab per column): larger slabs
+// stream better -- KKKV (12-byte rows) 4 -> 8 rows: 820 -> 584 us (3 x 15 KB slabs per
+// stage); key + WHERE column (8-byte rows) 8 -> 16: query 1 418 -> 391 us (KKV keeps 8:
+// 394 -> 414 with 16)
+#ifndef TOPK_ROW12_ITEMS
+#define TOPK_ROW12_ITEMS 8
+#endif
+#ifndef TOPK_ROW8_ITEMS
+#define TOPK_ROW8_ITEMS 16
+#endif
 #ifndef TOPK_FLUSH_ROWS
 #define TOPK_FLUSH_ROWS 2  // A/B: 3 -> 2 rows: k=256 362.5 -> 360.5 us, few-distinct 399 -> 394 (1 row: ties 1.5x slower)
 #endif
@@ -101,13 +111,15 @@ struct QCfg {
                                      ((Q & (kQRank | kQKey2)) ? 4 : 0) + ((Q & kQKey3) ? 4 : 0) +
                                      ((Q & kQPred) ? 4 : 0);
     static constexpr int kItems =
-        Q == 0 ? Cfg<Key>::kItems : (kRowBytes <= 8 ? 8 : 4);  // rows per consumer thread
+        Q == 0 ? Cfg<Key>::kItems
+               : (kRowBytes <= 8 ? ((Q & kQKey2) ? 8 : TOPK_ROW8_ITEMS)
+                                : (kRowBytes == 12 ? TOPK_ROW12_ITEMS : 4));
     static constexpr int kTileKeys = Q == 0 ? Cfg<Key>::kTileKeys : kNC * kItems;
     static constexpr int kVecPerThread = kItems / KeyTraits<Key>::kVec;
     static constexpr int kOffB = kTileKeys * static_cast<int>(sizeof(Key));  // column b
     static constexpr int kOffC = kOffB + ((Q & (kQRank | kQKey2)) ? kTileKeys * 4 : 0);  // key 3
     static constexpr int kOffP = kOffC + ((Q & kQKey3) ? kTileKeys * 4 : 0);  // predicate
-    static_assert(Q == 0 || kTileKeys * kRowBytes <= kTileBytes, "stage size");
+    static_assert(Q == 0 || kTileKeys * kRowBytes <= 2 * kTileBytes, "stage size");
     // ring: a query stage is TK rows of every column (<= one plain stage), so the ring
     // budget of the plain form holds more of them (up to kStagesMax)
     static constexpr int kSlotBytes = Q == 0 ? kTileBytes : (kTileKeys * kRowBytes + 127) / 128 * 128;
