@@ -350,7 +350,8 @@ constexpr int kReqFlush = 1, kReqRefresh = 2;
 // Shared state of one CTA.
 template <class E, class Key>
 struct CtaState {
-    int cnt;                   // survivors in buf[K ..)
+    int cnt;                   // bag entries buf[0 .. cnt) (reservations; see reserve())
+    int cnt_fail;              // min start of a failed reservation (INT_MAX: none); = cnt + 1
     int req;                   // collective requests (kReqFlush | kReqRefresh)
     int nflush;                // flushes done
     int last;                  // this CTA reduces all candidates
@@ -407,15 +408,31 @@ __device__ __forceinline__ Par<E96, Key> load_par(const CtaState<E96, Key>& st) 
     return st.par;
 }
 
-// Reserve `total` buffer entries (lane 31 of a warp): one atomicAdd; a reservation
-// that overshoots `limit` is undone and reported as -1.  Successful reservations are
-// always contiguous from 0 (a failed one leaves the counter above the limit until its
-// undo, so no success can start above it).
+// Reserve `total` buffer entries (lane 31 of a warp): one atomicAdd, or -1 if they
+// did not fit under `limit`.  A failure is NOT undone (add-then-undo is racy: with two
+// failed adds in flight, undoing one lets a third warp succeed ABOVE the other's phantom
+// entries -- a hole of stale entries in the bag (duplicates) and entries past the count
+// (lost); seen as ~4% wrong answers at f64, 2^24 keys, k = 1024).  Instead the counter
+// stays monotone until the flush, so the reservations are ordered by `old`: every one
+// after the first failure F starts at >= old_F + total_F > limit and fails too, every
+// one before F succeeded, and they fill exactly [0, old_F).  A failure records its
+// `old` in cnt[1] (CtaState::cnt_fail, atomicMin); the flush that every failure leads
+// to takes min(cnt, cnt_fail) as the bag size (bag_count()) and resets both.
 __device__ __forceinline__ int reserve(int* cnt, int total, int limit) {
+#ifdef TOPK_RESERVE_CAS  // (dev A/B: compare-and-swap form, ~10 us slower at k = 256)
+    int old = *reinterpret_cast<volatile int*>(cnt);
+    while (old + total <= limit) {
+        const int seen = atomicCAS(cnt, old, old + total);
+        if (seen == old) return old;
+        old = seen;
+    }
+    return -1;
+#else
     const int old = atomicAdd(cnt, total);
     if (old + total <= limit) return old;
-    atomicSub(cnt, total);
+    atomicMin(cnt + 1, old);
     return -1;
+#endif
 }
 
 // Warp-aggregated append of ITEMS candidate entries per thread (mask = which).
@@ -462,7 +479,11 @@ static __device__ unsigned long long g_stats[8];  // per translation unit (selec
 static __device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
 static __device__ __constant__ int c_trace_on;
 static __device__ __constant__ int c_dbg;
+#ifdef TOPK_DUPCHECK
+#define TOPK_STAT(i, v) ((void)0)
+#else
 #define TOPK_STAT(i, v) atomicAdd(&g_stats[i], static_cast<unsigned long long>(v))
+#endif
 __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
     unsigned long long t;
@@ -554,6 +575,32 @@ __device__ __forceinline__ void fold_bounds(CtaState<typename KeyTraits<Key>::E,
     }
     bound_set<Key, MIN>(st, tau);
 }
+
+#ifdef TOPK_DUPCHECK
+// (dev) count duplicate row ids in buf[0 .. cnt) into g_stats[slot]; order violations of
+// a sorted prefix into g_stats[oslot] (collective)
+template <class E>
+__device__ void dbg_check(const SBuf<E>& buf, int cnt, int slot, int sorted_n, int oslot) {
+    CSync::sync();
+    unsigned long long d = 0, o = 0;
+    for (int i = threadIdx.x; i < cnt; i += kNC) {
+        const E a = buf.ld(i);
+        if (a.is_sentinel()) continue;
+        for (int j = i + 1; j < cnt; ++j) {
+            const E b = buf.ld(j);
+            if (!b.is_sentinel() && b.lidx() == a.lidx()) ++d;
+        }
+        if (i + 1 < sorted_n && better(buf.ld(i + 1), a)) ++o;
+    }
+    if (d) atomicAdd(&g_stats[slot], d);
+    if (o) atomicAdd(&g_stats[oslot], o);
+    CSync::sync();
+}
+#define TOPK_DUP(...) dbg_check(__VA_ARGS__)
+static __device__ unsigned int g_tiles[1 << 16];
+#else
+#define TOPK_DUP(...) ((void)0)
+#endif
 
 enum FlushMode { kFlushStream = 0, kFlushFinal = 1 };
 
@@ -697,7 +744,8 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
     const int k = cx.k, K = cx.K;
     const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int c = static_cast<int>(blockIdx.x);
-    int cnt = st->cnt;
+    // (a failed reservation leaves cnt above the filled prefix; see reserve())
+    int cnt = st->cnt < st->cnt_fail ? st->cnt : st->cnt_fail;
     [[maybe_unused]] const int cnt0 = cnt;
     if (threadIdx.x == 0) trace(2);
     [[maybe_unused]] const long long t0 = clock64();
@@ -759,6 +807,7 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         take_bounds<Key, MIN>(st, cx, kth, publish);
         if (cnt > K) cnt = K;
     }
+    TOPK_DUP(buf, cnt, mode == kFlushStream ? 4 : 2, done ? 0 : (cnt < K ? cnt : K), 3);
     // every thread has read st (nflush, ties, limit) for this flush's decisions before
     // thread 0 updates it (racecheck: without this barrier a late warp could read the
     // incremented nflush and take a different `done` -- a divergent CSync)
@@ -770,6 +819,7 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         if (!done) TOPK_STAT(6, 1ull);
         if (tried && !done && publish) st->ties = 1;
         st->cnt = cnt;
+        st->cnt_fail = 0x7FFFFFFF;
         st->sorted_cnt = done ? -1 : cnt;
         st->nflush += 1;
         st->limit = next_limit(st->nflush, K, cx.Lp, st->ties);
@@ -1111,6 +1161,33 @@ __device__ __forceinline__ typename KeyTraits<Key>::E query_entry(const SelectPa
                            static_cast<uint32_t>(row));
 }
 
+
+// Tail: append ITEMS entries per thread (mask = which) to the bag, flushing (final mode)
+// whenever a warp's entries do not fit.  Collective over the consumer warps.
+template <class Key, bool MIN, int ITEMS>
+__device__ __forceinline__ void append_all(const SBuf<typename KeyTraits<Key>::E>& buf,
+                                           CtaState<typename KeyTraits<Key>::E, Key>* st,
+                                           const Ctx& cx,
+                                           const typename KeyTraits<Key>::E (&ents)[ITEMS],
+                                           uint32_t mask) {
+    using E = typename KeyTraits<Key>::E;
+    bool todo = true;
+    while (true) {
+        int vote = 0;
+        if (todo) {
+            if (__any_sync(0xFFFFFFFFu, mask != 0u)) {
+                const int old = append<E, ITEMS>(buf, &st->cnt, ents, mask, kCap);
+                todo = old < 0;
+                vote = todo ? 1 : 0;
+            } else {
+                todo = false;
+            }
+        }
+        if (!cbar_or(vote != 0)) break;
+        flush<Key, MIN>(buf, st, cx, kFlushFinal);
+    }
+}
+
 template <class Key, bool MIN, bool FILTER, int Q = 0>
 __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     using KT = KeyTraits<Key>;
@@ -1170,6 +1247,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         }
         fence_mbar_init();
         st.cnt = 0;
+        st.cnt_fail = 0x7FFFFFFF;
         st.req = 0;
         st.nflush = 0;
         st.sorted_cnt = -1;
@@ -1297,9 +1375,17 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             }
             if (__all_sync(0xFFFFFFFFu, mbar_try_wait(&full[slot], parity))) break;
         }
-        const uint32_t tile = st.tile[slot];
+        // (lane 0 -- the lane that arrives on empty[slot] -- reads the tile id: every
+        // read of st.tile[slot] is then ordered before the producer's next write of it by
+        // that arrive, which racecheck can see)
+        uint32_t tile = 0;
+        if (lane == 0) tile = st.tile[slot];
+        tile = __shfl_sync(0xFFFFFFFFu, tile, 0);
         if (tile == kEndTile) break;
         ++ntiles_done;
+#ifdef TOPK_DUPCHECK
+        if (tid == 0 && tile < (1u << 16)) atomicAdd(&g_tiles[tile], 1u);
+#endif
         const uint64_t tlo = static_cast<uint64_t>(tile) * TK;
         const uint32_t tlen = static_cast<uint32_t>(min(static_cast<uint64_t>(TK), p.body_n - tlo));
         const uint32_t lbase = static_cast<uint32_t>(p.head + tlo);
@@ -1340,6 +1426,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         for (int j = tid; j < K; j += kNC) buf.st(j, E::sentinel());
         CSync::sync();
     } else if (st.cnt != st.sorted_cnt) {
+        TOPK_DUP(buf, st.cnt, 1, 0, 3);
         flush<Key, MIN>(buf, &st, cx, kFlushFinal);
     }
 
@@ -1356,13 +1443,48 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (!st.last) return;
         __threadfence();
         if (tid == 0) trace(5);
-        // (1) Rank bound over the final runs (tail form of the flush bound): row j holds
-        // each run's 2^j-th best; the t-th largest (t = ceil(k / 2^j) <= G) bounds the
-        // global k-th best.  All loads in one parallel pass.
+        // (1) Stage the first kk entries of every other run in the idle ring (one L2 round
+        // trip for all of them; every run is sorted best first, so only a prefix of it can
+        // reach the global top-k).
         if (cx.nrows > TOPK_TAIL_ROWS) cx.nrows = TOPK_TAIL_ROWS;
+        constexpr int kEB = SBuf<E>::kBytes;
+        int kk = 1;
+        while (kk * 2 <= k && kk < 32) kk *= 2;  // largest power of two <= min(k, 32)
+        const int deep = 1 << (cx.j_lo + cx.nrows - 1);  // deepest rank-bound sample + 1
+        while (kk < deep && kk * 2 <= k) kk *= 2;
+        while (kk > 1 && ((static_cast<int>(G) * kk + 15) & ~15) * kEB > kStages * kSlot) kk >>= 1;
+        const int lk = __ffs(kk) - 1;
+        const int nst = static_cast<int>(G) << lk;
+        SBuf<E> stg;
+        stg.init(ring, (nst + 15) & ~15);
+        {
+            constexpr int U = 4;  // loads in flight per thread
+            for (int q0 = tid; q0 < nst; q0 += U * kNC) {
+                E v[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const int q = q0 + u * kNC;
+                    const int cc = q >> lk;
+                    v[u] = (q < nst && cc != static_cast<int>(c))
+                               ? cand.ld(static_cast<size_t>(cc) * k + (q & (kk - 1)))
+                               : E::sentinel();
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (q0 + u * kNC < nst) stg.st(q0 + u * kNC, v[u]);
+            }
+        }
+        CSync::sync();
+        // (2) Rank bound over the final runs (tail form of the flush bound): row j holds
+        // each run's 2^j-th best (from the staged prefixes where they lie inside them);
+        // the t-th largest (t = ceil(k / 2^j) <= G) bounds the global k-th best.
         for (int q = tid; q < cx.nrows * cx.G; q += kNC) {
             const int ji = cx.j_lo + q / cx.G, cc = q % cx.G;
-            scratch[q] = bound_word(cand.ld(static_cast<size_t>(cc) * k + (1u << ji) - 1u));
+            const int pos = (1 << ji) - 1;
+            const E e = (pos < kk && cc != static_cast<int>(c))
+                            ? stg.ld((cc << lk) + pos)
+                            : cand.ld(static_cast<size_t>(cc) * k + pos);
+            scratch[q] = bound_word(e);
         }
         CSync::sync();
         if (tid == 0) trace(8);
@@ -1370,12 +1492,14 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (tid == 0) trace(9);
         if (tid == 0) {
             E tb = from_bound_word<E>(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&hdr->tau_g)));
-            for (int ji = 0; ji < cx.J; ++ji) {
+            for (int ji = 0; ji < kPubRows; ++ji) {
                 const E b = from_bound_word<E>(st.best[ji]);
                 if (st.best[ji] != 0ull && better(b, tb)) tb = b;
             }
+            if (st.cnt_run >= k && better(buf.ld(k - 1), tb)) tb = buf.ld(k - 1);
             st.tau = tb;
             st.cnt = 0;
+            st.req = 0;
         }
         CSync::sync();
         const E tb = st.tau;
@@ -1383,102 +1507,87 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             const int own = st.cnt_run < k ? st.cnt_run : k;
             int q = 0;
             for (int j = tid; j < own; j += kNC) q += better(tb, buf.ld(j)) ? 0 : 1;
-            if (q) atomicAdd(&st.cnt, q);
+            q = __reduce_add_sync(0xFFFFFFFFu, q);
+            if (lane == 0 && q) atomicAdd(&st.cnt, q);
             CSync::sync();
             if (tid == 0) st.sorted_cnt = st.cnt;
             CSync::sync();
         }
         if (tid == 0) trace(11);
-        // (2) Every run is sorted best first, so only a prefix can be >= tb: append the
-        // qualifying entries of the first min(k, 32) of every other run (one parallel
-        // pass), then the rest of the runs whose 32nd entry still qualified (rare).
-        const int kk = k < 32 ? k : 32;
+        // (3) Append the qualifying staged entries; flag the runs whose last staged entry
+        // still qualified (their tails kk .. k are appended in (4)).
         __shared__ unsigned int s_more[(kGMax + 31) / 32];
-        for (int q = tid; q < (kGMax + 31) / 32; q += kNC) s_more[q] = 0u;
-        CSync::sync();
-        constexpr int CI = 11;  // one pass covers G * 32 <= 160 * 32 = 5120 <= 11 * 480
         __shared__ int s_flag_list[kGMax];
         __shared__ int s_nflag;
-        for (int phase = 0; phase < 2; ++phase) {
-            if (tid == 0) trace(12 + phase);
-            if (phase == 1) {  // compact the runs whose 32nd entry still qualified
-                if (kk >= k) break;
-                if (tid < 32) {  // warp 0: ballot-based compaction of the flag bits
-                    int nf = 0;
-                    for (int w0 = 0; w0 < (cx.G + 31) / 32; ++w0) {
-                        const int cc = w0 * 32 + tid;
-                        const bool f = cc < cx.G && ((s_more[w0] >> tid) & 1u);
-                        const uint32_t bal = __ballot_sync(0xFFFFFFFFu, f);
-                        if (f) s_flag_list[nf + __popc(bal & ((1u << tid) - 1u))] = cc;
-                        nf += __popc(bal);
+        for (int q = tid; q < (kGMax + 31) / 32; q += kNC) s_more[q] = 0u;
+        CSync::sync();
+        constexpr int CI = 11;
+        for (int q0 = 0; q0 < nst; q0 += CI * kNC) {
+            E ents[CI];
+            uint32_t mask = 0;
+#pragma unroll
+            for (int r = 0; r < CI; ++r) {
+                const int q = q0 + tid + r * kNC;
+                ents[r] = q < nst ? stg.ld(q) : E::sentinel();
+                if (!ents[r].is_sentinel() && !better(tb, ents[r])) {
+                    mask |= 1u << r;
+                    if ((q & (kk - 1)) == kk - 1 && kk < k) {
+                        const int cc = q >> lk;
+                        atomicOr(&s_more[cc >> 5], 1u << (cc & 31));
                     }
-                    if (tid == 0) s_nflag = nf;
                 }
-                CSync::sync();
             }
-            const int lo = phase == 0 ? 0 : kk;
-            const int span = phase == 0 ? kk : k - kk;
-            const int nruns = phase == 0 ? cx.G : s_nflag;
-            if (span <= 0 || nruns == 0) break;
-            // positions q = run_slot * spanp + j with spanp = next_pow2(span): shifts, no
-            // integer division (j >= span slots are skipped)
-            const int lsp = 32 - __clz(span - 1 > 0 ? span - 1 : 0);
-            const int total = nruns << lsp;
+            append_all<Key, MIN, CI>(buf, &st, cx, ents, mask);
+        }
+        CSync::sync();
+        if (tid == 0) trace(12);
+        // (4) The rest (positions kk .. k) of the flagged runs (rare: a run with more than
+        // kk entries in the global top-k).
+        if (kk < k) {
+            if (tid < 32) {  // warp 0: ballot-based compaction of the flag bits
+                int nf = 0;
+                for (int w0 = 0; w0 < (cx.G + 31) / 32; ++w0) {
+                    const int cc = w0 * 32 + tid;
+                    const bool f = cc < cx.G && ((s_more[w0] >> tid) & 1u);
+                    const uint32_t bal = __ballot_sync(0xFFFFFFFFu, f);
+                    if (f) s_flag_list[nf + __popc(bal & ((1u << tid) - 1u))] = cc;
+                    nf += __popc(bal);
+                }
+                if (tid == 0) s_nflag = nf;
+            }
+            CSync::sync();
+            const int span = k - kk;
+            const int lsp = 32 - __clz(span - 1 > 0 ? span - 1 : 0);  // next_pow2(span)
+            const int total = s_nflag << lsp;
             for (int q0 = 0; q0 < total; q0 += CI * kNC) {
                 E ents[CI];
                 uint32_t mask = 0;
-                // all loads first, unconditionally (invalid slots read entry 0 and are
-                // discarded) -- one L2 round trip instead of CI dependent ones
                 size_t at[CI];
                 bool ok[CI];
 #pragma unroll
                 for (int r = 0; r < CI; ++r) {
                     const int q = q0 + tid + r * kNC;
-                    const int qq = q < total ? q : 0;
-                    const int slot = qq >> lsp, j = qq & ((1 << lsp) - 1);
-                    const int cc = phase == 0 ? slot : s_flag_list[slot];
-                    ok[r] = q < total && j < span && cc != static_cast<int>(c);
-                    at[r] = ok[r] ? static_cast<size_t>(cc) * k + lo + j : 0;
+                    const int j = q & ((1 << lsp) - 1);
+                    ok[r] = q < total && j < span;
+                    at[r] = ok[r] ? static_cast<size_t>(s_flag_list[q >> lsp]) * k + kk + j : 0;
                 }
 #pragma unroll
                 for (int r = 0; r < CI; ++r) ents[r] = cand.ld(at[r]);
 #pragma unroll
                 for (int r = 0; r < CI; ++r) {
-                    const E e = ents[r];
-                    if (ok[r] && !e.is_sentinel() && !better(tb, e)) {
+                    if (ok[r] && !ents[r].is_sentinel() && !better(tb, ents[r]))
                         mask |= 1u << r;
-                        const int q = q0 + tid + r * kNC;
-                        const int j = lo + (q & ((1 << lsp) - 1));
-                        if (phase == 0 && j == kk - 1 && kk < k) {
-                            const int cc = q >> lsp;
-                            atomicOr(&s_more[cc >> 5], 1u << (cc & 31));
-                        }
-                    } else {
+                    else
                         ents[r] = E::sentinel();
-                    }
                 }
-                if (tid == 0) trace(14);
-                bool todo = true;
-                while (true) {
-                    int vote = 0;
-                    if (todo) {
-                        if (__any_sync(0xFFFFFFFFu, mask != 0u)) {
-                            const int old = append<E, CI>(buf, &st.cnt, ents, mask, kCap);
-                            todo = old < 0;
-                            vote = todo ? 1 : 0;
-                        } else {
-                            todo = false;
-                        }
-                    }
-                    if (tid == 0) trace(15);
-                    if (!cbar_or(vote != 0)) break;
-                    flush<Key, MIN>(buf, &st, cx, kFlushFinal);
-                }
+                append_all<Key, MIN, CI>(buf, &st, cx, ents, mask);
             }
             CSync::sync();
         }
         if (tid == 0) trace(10);
+        TOPK_DUP(buf, st.cnt, 5, 0, 3);
         if (st.cnt != st.sorted_cnt) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
+        TOPK_DUP(buf, k, 6, k, 3);
     }
     // ---- finalize: best first, original key bits, global index, payload ----
     for (int j = tid; j < k; j += kNC) {
@@ -1507,6 +1616,13 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (p.out_payload) p.out_payload[j] = p.payload[row];
     }
     if (tid == 0) trace(6);
+#ifdef TOPK_DUPCHECK
+    for (uint32_t q = tid; q < p.ntiles && q < (1u << 16); q += kNC) {
+        const unsigned int v = g_tiles[q];
+        if (v != 1u) atomicAdd(&g_stats[v == 0u ? 0 : 7], 1ull);
+        g_tiles[q] = 0u;
+    }
+#endif
     // leave the workspace zeroed for the next call (all other CTAs are done)
     for (int q = tid; q < kPubRows * static_cast<int>(G); q += kNC)
         cx.pub[static_cast<size_t>(q / G) * p.gmax + q % G] = 0ull;

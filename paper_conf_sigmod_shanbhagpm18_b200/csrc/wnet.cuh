@@ -126,10 +126,13 @@ __device__ __forceinline__ void wrebuild(E (&x)[R], int lane, uint32_t e0, int L
 // Entries per lane of a phase-A chunk: 16 (a 512-entry chunk) for 8-byte entries; 8 (256)
 // for the 12/16-byte entries of 64-bit codes and compound keys -- 16 of those would take
 // 48-64 registers per thread and spill under the kernel's 128-register cap.
+#ifndef TOPK_WIDE_R
+#define TOPK_WIDE_R 8
+#endif
 template <class E>
 struct WChunk {
-    static constexpr int R = sizeof(E) > 8 ? 8 : 16;
-    static constexpr int B = sizeof(E) > 8 ? 8 : 9;  // element bits inside a chunk
+    static constexpr int R = sizeof(E) > 8 ? TOPK_WIDE_R : 16;
+    static constexpr int B = R == 16 ? 9 : 8;  // element bits inside a chunk
 };
 
 // Register pass over 32 R-entry chunks of b[0..P): steps b = hi .. 0 with direction

@@ -175,3 +175,19 @@ def test_config5_2p32_two_chunks(cuda_device):
     for r in rows:
         h = datagen.generate("uniform", 1, "f32", seed=seed, base=int(r), n_total=n)
         assert host(h)[0] == host(xd[int(r):int(r) + 1])[0]
+
+
+@pytest.mark.parametrize("dt,lg,k", [("f64", 24, 1024), ("f32", 24, 2048), ("u32", 22, 1024)])
+def test_repeated_calls_identical(cuda_device, dt, lg, k):
+    """The kernel's schedule (which CTA claims which tiles, which one runs the tail) is
+    timing-dependent; the answer must not be.  Regression for the bag reservation race
+    (select.cuh reserve(): add-then-undo let a warp append above a failed warp's phantom
+    entries -- ~4% wrong answers at f64, 2^24, k = 1024): 60 calls, every one exact."""
+    n = 1 << lg
+    x = datagen.generate("uniform", n, dt, seed=n + 17, device=cuda_device)
+    ev, ei = oracle.topk(host(x), k, True)
+    bad = 0
+    for _ in range(60):
+        v, i = tk.topk(x, k, True)
+        bad += int(not (np.array_equal(i.cpu().numpy(), ei) and host(v).tobytes() == ev.tobytes()))
+    assert bad == 0, f"{bad}/60 calls wrong"
