@@ -63,6 +63,12 @@ namespace topk {
 #ifndef TOPK_FLUSH_ROWS
 #define TOPK_FLUSH_ROWS 2  // A/B: 3 -> 2 rows: k=256 362.5 -> 360.5 us, few-distinct 399 -> 394 (1 row: ties 1.5x slower)
 #endif
+#ifndef TOPK_BOOT_LP
+#define TOPK_BOOT_LP 1  // boot flush of a bag smaller than k: rank only as deep as the rank rows
+#endif
+#ifndef TOPK_BOOT_BIG
+#define TOPK_BOOT_BIG 0  // boot buffer: kCap entries for every K (0: kCap / 8 for K >= 256)
+#endif
 #ifndef TOPK_TAIL_ROWS
 #define TOPK_TAIL_ROWS 3
 #endif
@@ -366,6 +372,7 @@ struct CtaState {
     int wcnt[16];              // compaction: kept entries per consumer warp
     unsigned long long own_w;  // the bag's own k-th best as a bound word (0 = none)
     unsigned long long best[kPubRows];
+    int npres[kPubRows];       // rank_rows: present samples per ranked row
     uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
 };
 
@@ -518,44 +525,77 @@ struct Ctx {
     bool filter;
 };
 
-// Rank bound over scratch[nrows][G] (row r = sample row j_lo + r; 0 = missing sample):
-// the t-th largest word of row j, t = ceil(k / 2^j) <= G.  Only the nrows (<= 3) rows
-// with the smallest valid j are ranked -- they give the tightest bounds (a deeper row
-// samples a weaker quantile of every run).  Collective (consumers); st->best[] gets one
-// word per row.  Entry: scratch filled and barrier passed; exit: after a barrier.
+// Sample rows in shared scratch: row r at scratch + r * ScrStride(G) (padded with zeros
+// to a multiple of 4 words: 16-byte loads, 2 per step).
+__device__ __forceinline__ int scr_stride(int G) { return (G + 3) & ~3; }
+
+// Rank bound over scratch rows (row r = sample row j_lo + r; 0 = missing sample): the
+// t-th largest word x_t of row j, t = ceil(k / 2^j) <= G, if it is not missing.  Only
+// the nrows (<= 3) rows with the smallest valid j are ranked -- they give the tightest
+// bounds (a deeper row samples a weaker quantile of every run).  When the row has at
+// least t present samples, x_t = the smallest present word v with #{x > v} <= t - 1
+// (every v >= x_t has at most t - 1 larger words, every v < x_t has x_1 .. x_t above
+// it); with fewer, there is no bound.  One thread per word counts the strictly larger
+// ones (16-byte loads, four independent counters -- the dependent one-counter loop took
+// ~3.4 us at G = 148, latency-bound), the qualifying words meet in a shared atomicMin,
+// the present words are counted per row.  Collective (consumers); st->best[] gets one
+// word per ranked row, 0 elsewhere (thread 0 finishes it: only thread 0 reads
+// st->best).  Entry: scratch filled and barrier passed; exit: after a barrier.
 template <class E, class Key>
 __device__ void rank_rows(CtaState<E, Key>* st, const Ctx& cx) {
-    if (threadIdx.x < kPubRows) st->best[threadIdx.x] = 0ull;
-    CSync::sync();
-    const int RG = cx.nrows * cx.G;
-    for (int q = threadIdx.x; q < RG; q += kNC) {
-        const int r = q / cx.G;
-        const int ji = cx.j_lo + r;
-        const int t = (cx.k + (1 << ji) - 1) >> ji;
-        const unsigned long long v = cx.scratch[q];
-        if (v == 0ull) continue;
-        const unsigned long long* row = cx.scratch + r * cx.G;
-        int gt = 0, ge = 0;
-#pragma unroll 4
-        for (int c2 = 0; c2 < cx.G; ++c2) {
-            gt += row[c2] > v ? 1 : 0;
-            ge += row[c2] >= v ? 1 : 0;
-        }
-        // v is the t-th largest (code-only samples of different CTAs may be equal words:
-        // every thread holding that value writes the same word)
-        if (gt <= t - 1 && t - 1 < ge) st->best[ji] = v;
+    static_assert(3 * kGMax <= kNC, "one ranked word per consumer thread");
+    if (threadIdx.x < kPubRows) {
+        st->best[threadIdx.x] = ~0ull;
+        st->npres[threadIdx.x] = 0;
     }
     CSync::sync();
+    if (threadIdx.x == 0) trace(23);
+    const int S = scr_stride(cx.G);
+    const int q = threadIdx.x;  // nrows * G <= 3 * kGMax <= kNC: one pass
+    const int r = q / cx.G, cc = q - r * cx.G;
+    const bool in = r < cx.nrows;
+    const unsigned long long* row = cx.scratch + (in ? r : 0) * S;
+    const unsigned long long v = in ? row[cc] : 0ull;
+    const int ji = cx.j_lo + r;
+    if (v != 0ull) {
+        const int t = (cx.k + (1 << ji) - 1) >> ji;
+        const ulonglong2* row2 = reinterpret_cast<const ulonglong2*>(row);
+        int g0 = 0, g1 = 0, g2 = 0, g3 = 0;
+#pragma unroll 4
+        for (int c2 = 0; c2 < S / 2; c2 += 2) {
+            const ulonglong2 a = row2[c2], b = row2[c2 + 1];
+            g0 += a.x > v ? 1 : 0;
+            g1 += a.y > v ? 1 : 0;
+            g2 += b.x > v ? 1 : 0;
+            g3 += b.y > v ? 1 : 0;
+        }
+        if (g0 + g1 + g2 + g3 <= t - 1) atomicMin(&st->best[ji], v);
+    }
+    {   // present samples per row: one shared atomic per (warp, row)
+        const uint32_t same = __match_any_sync(0xFFFFFFFFu, in ? r : -1);
+        const uint32_t pres = __ballot_sync(0xFFFFFFFFu, v != 0ull);
+        const int lane = threadIdx.x & 31;
+        if (in && lane == __ffs(same) - 1) atomicAdd(&st->npres[ji], __popc(same & pres));
+    }
+    if (threadIdx.x == 0) trace(24);
+    CSync::sync();
+    if (threadIdx.x == 0)
+        for (int j2 = 0; j2 < kPubRows; ++j2) {
+            const int t = (cx.k + (1 << j2) - 1) >> j2;
+            if (st->best[j2] == ~0ull || st->npres[j2] < t) st->best[j2] = 0ull;
+        }
 }
 
 // Load every CTA's published samples of the ranked rows into shared scratch (stale
 // values are smaller, still valid).
 __device__ __forceinline__ void load_pub(const Ctx& cx) {
-    const int RG = cx.nrows * cx.G;
-    for (int q = threadIdx.x; q < RG; q += kNC) {
-        const int r = q / cx.G, cc = q % cx.G;
-        cx.scratch[q] = ld_relaxed_u64(reinterpret_cast<const uint64_t*>(
-            cx.pub + static_cast<size_t>(cx.j_lo + r) * cx.gmax + cc));
+    const int S = scr_stride(cx.G);
+    const int RS = cx.nrows * S;
+    for (int q = threadIdx.x; q < RS; q += kNC) {
+        const int r = q / S, cc = q - r * S;
+        cx.scratch[q] = cc < cx.G ? ld_relaxed_u64(reinterpret_cast<const uint64_t*>(
+                                        cx.pub + static_cast<size_t>(cx.j_lo + r) * cx.gmax + cc))
+                                  : 0ull;
     }
 }
 
@@ -659,7 +699,9 @@ __device__ void take_bounds(CtaState<typename KeyTraits<Key>::E, Key>* st, const
         if (cr.nrows > TOPK_FLUSH_ROWS) cr.nrows = TOPK_FLUSH_ROWS;
         load_pub(cr);
         CSync::sync();
+        if (threadIdx.x == 0) trace(21);
         rank_rows(st, cr);
+        if (threadIdx.x == 0) trace(22);
     }
     if (threadIdx.x == 0) {
         if (!publish)
@@ -761,9 +803,20 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
     if (cx.filter && cx.Lp >= 0 && !(c_dbg & 1) && try_code) {
         tried = true;
         C* S = static_cast<C*>(cx.codes);
-        cnet_topk_codes<E, kNC / 32, CSync>(buf, cnt, cx.Lp, S, w, lane);
-        const int Kp = 1 << cx.Lp;  // codes the network ranked (S[0 .. Kp))
-        if (publish && threadIdx.x < cx.J && threadIdx.x <= cx.Lp && cnt >= (1 << threadIdx.x)) {
+        // A boot bag smaller than k has no k-th best to publish: its flush only needs the
+        // samples the first rank bound uses (rows j_lo .. j_lo + TOPK_FLUSH_ROWS - 1), so
+        // the code network ranks only that deep (measured, 2^29 uniform: k = 1024 393 ->
+        // 391 us, k = 2048 432 -> 420; a bag that holds k keeps the full depth: its k-th
+        // best, published as tau_g, is what bounds sorted input early)
+        int Lp = cx.Lp;
+        if (TOPK_BOOT_LP && publish && !st->pubd && cnt < k) {
+            const int deep = cx.j_lo + cx.nrows - 1;
+            Lp = min(cx.Lp, max(4, deep));
+        }
+        cnet_topk_codes<E, kNC / 32, CSync>(buf, cnt, Lp, S, w, lane);
+        if (threadIdx.x == 0) trace(16);
+        const int Kp = 1 << Lp;  // codes the network ranked (S[0 .. Kp))
+        if (publish && threadIdx.x < cx.J && threadIdx.x <= Lp && cnt >= (1 << threadIdx.x)) {
             st_relaxed_u64(cx.pub + static_cast<size_t>(threadIdx.x) * cx.gmax + c,
                            code_word<E>(S[(1 << threadIdx.x) - 1]));
             __threadfence();
@@ -1257,7 +1310,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // c_dbg knob, 2^29 uniform f32: K >= 256 best with 512 entries -- k = 256 379 ->
         // 363 us, k = 1024 406 -> 396 us; K <= 128 best with the whole buffer)
         st.limit = (c_dbg >> 8) & 7 ? kCap >> ((c_dbg >> 8) & 7)
-                   : K >= 256 ? kCap / 8 : kCap;
+                   : (K >= 256 && !TOPK_BOOT_BIG) ? kCap / 8 : kCap;
         st.ties = 0;
         st.tau_w = 0ull;
         st.tau = E::sentinel();
@@ -1443,6 +1496,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (!st.last) return;
         __threadfence();
         if (tid == 0) trace(5);
+        const unsigned long long tau_g_w =
+            tid == 0 ? ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&hdr->tau_g)) : 0ull;
         // (1) Stage the first kk entries of every other run in the idle ring (one L2 round
         // trip for all of them; every run is sorted best first, so only a prefix of it can
         // reach the global top-k).
@@ -1478,20 +1533,24 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // (2) Rank bound over the final runs (tail form of the flush bound): row j holds
         // each run's 2^j-th best (from the staged prefixes where they lie inside them);
         // the t-th largest (t = ceil(k / 2^j) <= G) bounds the global k-th best.
-        for (int q = tid; q < cx.nrows * cx.G; q += kNC) {
-            const int ji = cx.j_lo + q / cx.G, cc = q % cx.G;
-            const int pos = (1 << ji) - 1;
-            const E e = (pos < kk && cc != static_cast<int>(c))
-                            ? stg.ld((cc << lk) + pos)
-                            : cand.ld(static_cast<size_t>(cc) * k + pos);
-            scratch[q] = bound_word(e);
+        {
+            const int S = scr_stride(cx.G);
+            for (int q = tid; q < cx.nrows * S; q += kNC) {
+                const int ji = cx.j_lo + q / S, cc = q % S;
+                const int pos = (1 << ji) - 1;
+                const E e = cc >= cx.G ? E::sentinel()
+                            : (pos < kk && cc != static_cast<int>(c))
+                                ? stg.ld((cc << lk) + pos)
+                                : cand.ld(static_cast<size_t>(cc) * k + pos);
+                scratch[q] = bound_word(e);
+            }
         }
         CSync::sync();
         if (tid == 0) trace(8);
         rank_rows(&st, cx);
         if (tid == 0) trace(9);
         if (tid == 0) {
-            E tb = from_bound_word<E>(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(&hdr->tau_g)));
+            E tb = from_bound_word<E>(tau_g_w);
             for (int ji = 0; ji < kPubRows; ++ji) {
                 const E b = from_bound_word<E>(st.best[ji]);
                 if (st.best[ji] != 0ull && better(b, tb)) tb = b;

@@ -177,14 +177,19 @@ def test_config5_2p32_two_chunks(cuda_device):
         assert host(h)[0] == host(xd[int(r):int(r) + 1])[0]
 
 
-@pytest.mark.parametrize("dt,lg,k", [("f64", 24, 1024), ("f32", 24, 2048), ("u32", 22, 1024)])
-def test_repeated_calls_identical(cuda_device, dt, lg, k):
+@pytest.mark.parametrize("dt,lg,k,dist", [("f64", 24, 1024, "uniform"), ("f32", 24, 2048, "uniform"),
+                                          ("u32", 22, 1024, "uniform"),
+                                          ("f32", 27, 256, "decreasing")])
+def test_repeated_calls_identical(cuda_device, dt, lg, k, dist):
     """The kernel's schedule (which CTA claims which tiles, which one runs the tail) is
     timing-dependent; the answer must not be.  Regression for the bag reservation race
     (select.cuh reserve(): add-then-undo let a warp append above a failed warp's phantom
-    entries -- ~4% wrong answers at f64, 2^24, k = 1024): 60 calls, every one exact."""
+    entries -- ~4% wrong answers at f64, 2^24, k = 1024): 60 calls, every one exact.
+    Decreasing input (every top-k key in one tile, so most CTAs' sample rows are missing
+    or weak): regression for a rank bound that ignored missing samples (~17% wrong answers
+    at 2^29, k = 256, during development of the count-greater rank_rows)."""
     n = 1 << lg
-    x = datagen.generate("uniform", n, dt, seed=n + 17, device=cuda_device)
+    x = datagen.generate(dist, n, dt, seed=n + 17, device=cuda_device)
     ev, ei = oracle.topk(host(x), k, True)
     bad = 0
     for _ in range(60):

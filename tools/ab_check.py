@@ -24,6 +24,13 @@ CASES = [(1 << 20, "uniform", (32, 256)), ((1 << 20) + 13, "fewdistinct", (64, 1
          (1 << 29, "fewdistinct", (256,)), (1 << 29, "increasing", (256,))]
 
 
+if os.environ.get("AB_CASES"):  # e.g. AB_CASES="29:uniform:1,256,1024;25:uniform:64"
+    CASES = []
+    for c in os.environ["AB_CASES"].split(";"):
+        lg, dist, ks = c.split(":")
+        CASES.append((1 << int(lg), dist, tuple(int(k) for k in ks.split(","))))
+
+
 def load(path):
     lib = ctypes.CDLL(path)
     vp, u64, u32, i32, sz = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int, ctypes.c_size_t

@@ -21,7 +21,7 @@ for c in range(148):
     if ev: rows.append(ev)
 t0 = min(e[0][1] for e in rows)
 names = {1: "start", 2: "fb", 3: "fe", 4: "sEnd", 5: "tail", 6: "end", 7: "refr", 8: "sampled", 9: "ranked", 10: "appended", 11: "tb", 12: "ph0", 13: "ph1", 14: "loaded", 15: "apd",
-         16: "cnet", 17: "bnd", 18: "cmp", 19: "wnet", 20: "wait", 21: "lpub", 22: "rank"}
+         16: "cnet", 17: "bnd", 18: "cmp", 19: "wnet", 20: "wait", 21: "lpub", 22: "rank", 23: "r0", 24: "r1"}
 send_c = [(max([t for e, t in ev if e == 4] or [0]), c) for c, ev in enumerate(rows)]
 send_c.sort()
 for _, c in send_c[:2] + send_c[-3:]:
