@@ -493,14 +493,21 @@ static __device__ __constant__ int c_dbg;
 #endif
 __device__ __forceinline__ void trace(int ev) {
     if (!c_trace_on || blockIdx.x >= kTraceCtas) return;
-    unsigned long long t;
-    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-    // (the event count lives in shared memory: a stamp costs one fire-and-forget store)
+    // stamps are SM clock cycles (a %globaltimer read costs ~1 us and inflated every
+    // interval it bracketed); the CTA's first stamp also records (globaltimer, clock)
+    // in the last two slots, which align the CTAs (tools/trace.py)
+    const unsigned long long t = clock64();
     unsigned long long* row = g_trace[blockIdx.x];
     __shared__ int s_trace_n;
-    if (ev == 1) s_trace_n = 0;
+    if (ev == 1) {
+        s_trace_n = 0;
+        unsigned long long g;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(g));
+        row[kTraceLen - 1] = g;
+        row[kTraceLen - 2] = t;
+    }
     const int n = s_trace_n;
-    if (n + 1 < kTraceLen) {
+    if (n + 3 < kTraceLen) {
         row[n + 1] = (static_cast<unsigned long long>(ev) << 56) | (t & 0x00FFFFFFFFFFFFFFull);
         row[0] = static_cast<unsigned long long>(n + 1);
         s_trace_n = n + 1;
@@ -1596,7 +1603,9 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                     }
                 }
             }
+            if (tid == 0) trace(25);
             append_all<Key, MIN, CI>(buf, &st, cx, ents, mask);
+            if (tid == 0) trace(26);
         }
         CSync::sync();
         if (tid == 0) trace(12);
@@ -1644,6 +1653,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             CSync::sync();
         }
         if (tid == 0) trace(10);
+        if (tid == 0) trace(32 + min(st.cnt >> 6, 31));
         TOPK_DUP(buf, st.cnt, 5, 0, 3);
         if (st.cnt != st.sorted_cnt) flush<Key, MIN>(buf, &st, cx, kFlushFinal);
         TOPK_DUP(buf, k, 6, k, 3);

@@ -16,12 +16,16 @@ buf = np.zeros((160, 64), dtype=np.uint64)
 lib.topk_debug_trace(0, buf.ctypes.data_as(ctypes.c_void_p))
 t0 = None
 rows = []
+GHZ = float(os.environ.get("TRACE_GHZ", "1.965"))  # stamps are SM clocks (select.cuh trace)
 for c in range(148):
-    m = int(buf[c, 0]); ev = [(int(v) >> 56, int(v) & ((1 << 56) - 1)) for v in buf[c, 1:m + 1]]
+    m = int(buf[c, 0])
+    g0, c0 = int(buf[c, 63]), int(buf[c, 62]) & ((1 << 56) - 1)
+    ev = [(int(v) >> 56, g0 + ((int(v) & ((1 << 56) - 1)) - c0) / GHZ) for v in buf[c, 1:m + 1]]
     if ev: rows.append(ev)
 t0 = min(e[0][1] for e in rows)
 names = {1: "start", 2: "fb", 3: "fe", 4: "sEnd", 5: "tail", 6: "end", 7: "refr", 8: "sampled", 9: "ranked", 10: "appended", 11: "tb", 12: "ph0", 13: "ph1", 14: "loaded", 15: "apd",
-         16: "cnet", 17: "bnd", 18: "cmp", 19: "wnet", 20: "wait", 21: "lpub", 22: "rank", 23: "r0", 24: "r1"}
+         16: "cnet", 17: "bnd", 18: "cmp", 19: "wnet", 20: "wait", 21: "lpub", 22: "rank", 23: "r0", 24: "r1", 25: "mask", 26: "apd1"}
+for _e in range(32, 64): names[_e] = f"cnt{(_e - 32) * 64}+"
 send_c = [(max([t for e, t in ev if e == 4] or [0]), c) for c, ev in enumerate(rows)]
 send_c.sort()
 for _, c in send_c[:2] + send_c[-3:]:
