@@ -66,8 +66,8 @@ namespace topk {
 #ifndef TOPK_BOOT_LP
 #define TOPK_BOOT_LP 1  // boot flush of a bag smaller than k: rank only as deep as the rank rows
 #endif
-#ifndef TOPK_BOOT_BIG
-#define TOPK_BOOT_BIG 0  // boot buffer: kCap entries for every K (0: kCap / 8 for K >= 256)
+#ifndef TOPK_BOOT_SMALL_K
+#define TOPK_BOOT_SMALL_K 256  // K from which the boot buffer is kCap / 8 entries (else kCap)
 #endif
 #ifndef TOPK_TAIL_ROWS
 #define TOPK_TAIL_ROWS 3
@@ -765,8 +765,10 @@ __device__ int compact_bag(const SBuf<E>& buf, int cnt, E tau, int* s_w) {
 // one buffer per CTA only) and the rank bound tightens early.  A stream flush always
 // leaves at most half of the next limit (progress: a warp appends <= 512 at a time).
 __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
-    // (K = 256: 2K = 512 measured 6 us faster than 1024; other K: no difference)
-    const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3)) : K == 256 ? 512 : TOPK_LIMIT2;
+    // (K = 256: 512 measured 6 us faster than 1024, K = 128: 360 -> 354 us; other K: 512
+    // no better, 2048 slower)
+    const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3))
+                   : (K == 128 || K == 256) ? 512 : TOPK_LIMIT2;
     // Tie-heavy bags (the code path failed on equal keys) flush exactly at a small size:
     // every CTA meets the ties at about the same time and a 4096-entry exact flush idles
     // the HBM for ~20 us.  Progress: room for a warp's largest append (32 lanes x 16
@@ -1317,7 +1319,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // c_dbg knob, 2^29 uniform f32: K >= 256 best with 512 entries -- k = 256 379 ->
         // 363 us, k = 1024 406 -> 396 us; K <= 128 best with the whole buffer)
         st.limit = (c_dbg >> 8) & 7 ? kCap >> ((c_dbg >> 8) & 7)
-                   : (K >= 256 && !TOPK_BOOT_BIG) ? kCap / 8 : kCap;
+                   : (K >= TOPK_BOOT_SMALL_K) ? kCap / 8 : kCap;
         st.ties = 0;
         st.tau_w = 0ull;
         st.tau = E::sentinel();
