@@ -334,12 +334,22 @@ def size_sweep(tk, datagen, stream, torch, peak, k=64):
         for _ in range(3):
             f()
         if lg <= 25:
-            per = []
+            # flush, event, launch, event -- enqueued without a host synchronisation in
+            # between: the ~70 us flush keeps the GPU busy while the host enqueues the
+            # launch, so the events bracket the device time only (a synchronize before
+            # the first event let ~25 us of Python call overhead into the interval)
+            torch.cuda.synchronize()
+            evs = []
             for _ in range(10):
                 flush_l2()
-                _, t = time_steps(f, 1, stream, torch, per_step=True)
-                per.append(t[0])
-            us = statistics.median(per) * 1e3
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                f()
+                e1.record(stream)
+                evs.append((e0, e1))
+            torch.cuda.synchronize()
+            us = statistics.median(a.elapsed_time(b) for a, b in evs) * 1e3
             l2 = "flushed"
         else:
             _, per = time_steps(f, 10, stream, torch, per_step=True)

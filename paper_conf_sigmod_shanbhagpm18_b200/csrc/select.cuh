@@ -69,6 +69,9 @@ namespace topk {
 #ifndef TOPK_BOOT_SMALL_K
 #define TOPK_BOOT_SMALL_K 256  // K from which the boot buffer is kCap / 8 entries (else kCap)
 #endif
+#ifndef TOPK_BOOT_SAMPLE
+#define TOPK_BOOT_SAMPLE 1  // boot bag = the best key of each consumer thread's share of tile 0
+#endif
 #ifndef TOPK_TAIL_ROWS
 #define TOPK_TAIL_ROWS 3
 #endif
@@ -351,7 +354,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 }
 
 constexpr uint32_t kEndTile = 0xFFFFFFFFu;
-constexpr int kReqFlush = 1, kReqRefresh = 2;
+constexpr int kReqFlush = 1, kReqRefresh = 2, kReqBoot = 4;
 
 // Shared state of one CTA.
 template <class E, class Key>
@@ -373,6 +376,8 @@ struct CtaState {
     unsigned long long own_w;  // the bag's own k-th best as a bound word (0 = none)
     unsigned long long best[kPubRows];
     int npres[kPubRows];       // rank_rows: present samples per ranked row
+    int nx;                    // kBoot, CTA 0: extras kept aside until the boot flush
+    unsigned long long xent[8];
     uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
 };
 
@@ -485,8 +490,13 @@ constexpr int kTraceCtas = 160, kTraceLen = 64;
 static __device__ unsigned long long g_stats[8];  // per translation unit (select_inst.cuh)
 static __device__ unsigned long long g_trace[kTraceCtas][kTraceLen];
 static __device__ __constant__ int c_trace_on;
-static __device__ __constant__ int c_dbg;
-#ifdef TOPK_DUPCHECK
+static __device__ __constant__ int c_dbg_sym;  // topk_debug_flags
+#ifdef TOPK_LIGHT  // -DTOPK_DEBUG -DTOPK_LIGHT: trace stamps only (no counters, no knobs)
+constexpr int c_dbg = 0;
+#else
+#define c_dbg c_dbg_sym
+#endif
+#if defined(TOPK_DUPCHECK) || defined(TOPK_LIGHT)
 #define TOPK_STAT(i, v) ((void)0)
 #else
 #define TOPK_STAT(i, v) atomicAdd(&g_stats[i], static_cast<unsigned long long>(v))
@@ -530,6 +540,7 @@ struct Ctx {
     int Lp;           // code network size log2 K' (K' = min(max(K, 16), 512)); -1: not used
     void* codes;      // shared: code-network scratch (8 x K' codes)
     bool filter;
+    bool boot;        // the kernel runs the boot sample (kBoot)
 };
 
 // Sample rows in shared scratch: row r at scratch + r * ScrStride(G) (padded with zeros
@@ -764,7 +775,10 @@ __device__ int compact_bag(const SBuf<E>& buf, int cnt, E tau, int* s_w) {
 // cheap second flush soon publishes samples of many more keys (the boot samples cover
 // one buffer per CTA only) and the rank bound tightens early.  A stream flush always
 // leaves at most half of the next limit (progress: a warp appends <= 512 at a time).
-__device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
+#ifndef TOPK_L2_BOOT
+#define TOPK_L2_BOOT 128
+#endif
+__device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties, bool boot = false) {
     // (K = 256: 512 measured 6 us faster than 1024, K = 128: 360 -> 354 us; other K: 512
     // no better, 2048 slower)
     const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3))
@@ -774,6 +788,11 @@ __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties) {
     // the HBM for ~20 us.  Progress: room for a warp's largest append (32 lanes x 16
     // keys = 512) on top of the K entries an exact flush keeps.
     if (ties) return max(max(2 * K, K + 512), kCap >> 3);
+    // After a boot sample (boot_sample) the bound already stands on a 16x larger sample:
+    // the survivors arrive ~16x slower, so the second flush -- the one that publishes
+    // samples of many tiles -- comes at a much smaller bag.  (Progress: that flush makes
+    // nflush 2, whose limit is kCap.)
+    if (boot && nflush == 1 && Lp >= 0 && !(c_dbg & 4)) return TOPK_L2_BOOT;
     return (nflush == 1 && Lp >= 0 && !(c_dbg & 4)) ? max(l2, 2 * K) : kCap;
 }
 
@@ -842,7 +861,10 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         // (equal codes): finish exactly, and skip the code path from now on
         const bool weak = heavy || (cnt > 2 * K && 2 * cnt > cnt0);
         done = mode == kFlushStream && !weak &&
-               cnt <= next_limit(st->nflush + 1, K, cx.Lp, 0) / 2;
+               cnt <= next_limit(st->nflush + 1, K, cx.Lp, 0, cx.boot) / 2;
+        // (the boot sample's bag is emptied after this flush: no exact pass unless the
+        // code bound was defeated by ties)
+        if (st->req & kReqBoot) done = !weak;
     }
     if (!done) {
         int P = next_pow2_i(cnt);
@@ -880,11 +902,19 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         TOPK_STAT(2, static_cast<unsigned long long>(clock64() - t0));
         if (!done) TOPK_STAT(6, 1ull);
         if (tried && !done && publish) st->ties = 1;
+        if constexpr (std::is_same<E, E32>::value) {
+            if (st->req & kReqBoot) {  // boot sample flushed (boot_sample): empty the bag
+                for (int q = 0; q < st->nx; ++q) buf.st(q, E32{st->xent[q]});  // (CTA 0)
+                cnt = st->nx;
+                done = true;
+                if (st->tau_w != 0ull) st->tau_w -= 1ull;  // keep >= the bound on re-read keys
+            }
+        }
         st->cnt = cnt;
         st->cnt_fail = 0x7FFFFFFF;
         st->sorted_cnt = done ? -1 : cnt;
         st->nflush += 1;
-        st->limit = next_limit(st->nflush, K, cx.Lp, st->ties);
+        st->limit = next_limit(st->nflush, K, cx.Lp, st->ties, cx.boot);
         st->req = 0;
         trace(3);
     }
@@ -904,6 +934,39 @@ __device__ void refresh(CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx
         st->req = 0;
         trace(7);
     }
+    CSync::sync();
+}
+
+// Boot sample (kBoot): each consumer thread appends the best entry among its keys of the
+// first tile (positions as in consume_tile) and requests a flush, which the consumers
+// run as their next collective (one flush call site: a second inlined copy of flush()
+// spilled ~280 bytes per thread under the 128-register cap); that flush publishes the bag's
+// samples and its k-th best (real entries of the input, so every bound derived from them
+// is valid) and then empties the bag (kReqBoot) -- the tile is consumed next, against the
+// boot bound weakened by one entry step: an entry EQUAL to the bound (its own k-th best,
+// or its own sample coming back as the rank bound) was a bag entry and is now a new key
+// again, and new keys must only be strictly better than the bound to be appended.
+// Collective (consumers); the bag is empty on entry.
+template <class Key, bool MIN>
+__device__ void boot_sample(const unsigned char* slot_data, uint32_t tlen, uint32_t lbase,
+                            const SBuf<E32>& buf, CtaState<E32, Key>* st) {
+    using KT = KeyTraits<Key>;
+    constexpr int VEC = KT::kVec, ITEMS = Cfg<Key>::kItems;
+    const Key* sk = reinterpret_cast<const Key*>(slot_data);
+    const int tid = threadIdx.x;
+    E32 m = E32::sentinel();
+#pragma unroll
+    for (int q = 0; q < ITEMS; ++q) {
+        const uint32_t pos = static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
+        if (pos < tlen) {
+            const E32 e = E32::make(KT::template code<MIN>(sk[pos]), lbase + pos);
+            if (better(e, m)) m = e;
+        }
+    }
+    const E32 ents[1] = {m};
+    append<E32, 1>(buf, &st->cnt, ents, m.is_sentinel() ? 0u : 1u, kCap);  // <= kNC entries
+    CSync::sync();
+    if (threadIdx.x == 0) st->req |= kReqFlush | kReqBoot;  // flushed by the collective
     CSync::sync();
 }
 
@@ -1260,6 +1323,11 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     constexpr int kStages = QC::kStages;
     constexpr int kSlot = QC::kSlotBytes;
     static_assert(Q == 0 || FILTER, "query forms run in filter mode");
+    // Boot sample (plain 32-bit-key form): the boot bag is the best key of each consumer
+    // thread's share of the first tile (480 entries, each the best of 16 keys) instead of
+    // the tile's first keys -- the same flush, a 16x larger sample behind its bound.  The
+    // bag is then emptied and the tile consumed as usual.
+    constexpr bool kBoot = FILTER && Q == 0 && std::is_same<E, E32>::value && TOPK_BOOT_SAMPLE;
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ CtaState<E, Key> st;
@@ -1297,6 +1365,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         cx.nrows = cx.J - cx.j_lo < maxrows ? cx.J - cx.j_lo : maxrows;
     }
     cx.filter = FILTER;
+    cx.boot = kBoot;
     // K > 512: the code network still gives the bag's 2^j-th best codes for j <= 9,
     // whose cross-CTA rank bound bounds the global k-th best (t = ceil(k / 2^j) <= G)
     cx.Lp = FILTER ? (K < 16 ? 4 : min(__ffs(K) - 1, 9)) : -1;
@@ -1309,6 +1378,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         }
         fence_mbar_init();
         st.cnt = 0;
+        st.nx = 0;
         st.cnt_fail = 0x7FFFFFFF;
         st.req = 0;
         st.nflush = 0;
@@ -1319,14 +1389,15 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         // c_dbg knob, 2^29 uniform f32: K >= 256 best with 512 entries -- k = 256 379 ->
         // 363 us, k = 1024 406 -> 396 us; K <= 128 best with the whole buffer)
         st.limit = (c_dbg >> 8) & 7 ? kCap >> ((c_dbg >> 8) & 7)
-                   : (K >= TOPK_BOOT_SMALL_K) ? kCap / 8 : kCap;
+                   : (K >= TOPK_BOOT_SMALL_K && !kBoot) ? kCap / 8 : kCap;
         st.ties = 0;
         st.tau_w = 0ull;
         st.tau = E::sentinel();
         st.par = make_par<Key, MIN>(E::sentinel());
     }
-    // Extras: the unaligned head and the sub-16-byte tail, appended by CTA 0.
-    if (c == 0) {
+    // Extras: the unaligned head and the sub-16-byte tail, appended by CTA 0 to an empty
+    // bag (at the start, or after the boot sample's flush).
+    auto append_extras = [&]() {
         const uint64_t tail0 = p.head + p.body_n;
         const int nextra = static_cast<int>(p.head + (p.n - tail0));
         if constexpr (Q == 0) {
@@ -1343,6 +1414,20 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             const uint32_t bal = __ballot_sync(0xFFFFFFFFu, ok);
             if (ok) buf.st(__popc(bal & ((1u << tid) - 1u)), query_entry<Key, MIN, Q>(p, keys, row));
             if (tid == 0) st.cnt = __popc(bal);
+        }
+    };
+    if (c == 0) {
+        if constexpr (kBoot) {  // kept aside: the boot flush empties the bag, then adds them
+            const uint64_t tail0 = p.head + p.body_n;
+            const int nextra = static_cast<int>(p.head + (p.n - tail0));
+            if (tid < nextra) {
+                const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
+                                                                     : tail0 + (tid - p.head);
+                st.xent[tid] = E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row)).v;
+            }
+            if (tid == 0) st.nx = nextra;
+        } else {
+            append_extras();
         }
     }
     __syncthreads();
@@ -1423,6 +1508,28 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             refresh<Key, MIN>(&st, cx);
     };
     uint32_t ntiles_done = 0;
+    if constexpr (kBoot) {
+        // boot sample: wait for the first slot, append each thread's best key of it and
+        // request its flush -- the main loop's first wait runs that flush as a collective
+        // and then consumes the same tile.  (A CTA without tiles appends the extras here;
+        // otherwise the boot flush does, after emptying the bag.)
+        while (!__all_sync(0xFFFFFFFFu, mbar_try_wait(&full[0], 0u))) {
+        }
+        uint32_t tile = 0;
+        if (lane == 0) tile = st.tile[0];
+        tile = __shfl_sync(0xFFFFFFFFu, tile, 0);
+        if (tile != kEndTile) {
+            boot_sample<Key, MIN>(ring, static_cast<uint32_t>(min(static_cast<uint64_t>(TK),
+                                                                  p.body_n - static_cast<uint64_t>(tile) * TK)),
+                                  static_cast<uint32_t>(p.head + static_cast<uint64_t>(tile) * TK), buf, &st);
+        } else {
+            if (tid == 0) {
+                for (int q = 0; q < st.nx; ++q) buf.st(q, E32{st.xent[q]});
+                st.cnt = st.nx;
+            }
+            CSync::sync();
+        }
+    }
 #pragma unroll 1
     for (uint32_t s = 0;; ++s) {
         const int slot = static_cast<int>(s % kStages);

@@ -50,7 +50,7 @@ int TOPK_CAT(TOPK_INST_FN, _debug)(int op, void* host, int arg) {
             return cudaMemcpyToSymbol(g_stats, z, sizeof(z)) == cudaSuccess ? 0 : -1;
         }
         case kDbgFlags:
-            return cudaMemcpyToSymbol(c_dbg, &arg, sizeof(int)) == cudaSuccess ? 0 : -1;
+            return cudaMemcpyToSymbol(c_dbg_sym, &arg, sizeof(int)) == cudaSuccess ? 0 : -1;
         case kDbgTraceRead:  // host: u64[kTraceCtas][kTraceLen]
             return cudaMemcpyFromSymbol(host, g_trace, sizeof(g_trace)) == cudaSuccess ? 0 : -1;
         case kDbgTraceSet: {  // clear, then enable (arg = 1) or disable

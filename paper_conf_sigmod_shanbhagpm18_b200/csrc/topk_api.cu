@@ -611,13 +611,17 @@ topk_status_t topk_merge_sorted(topk_dtype_t dtype, const void* cand_keys,
 /* Debug (not in topk.h's stable surface): read / reset the device counters of
  * select_kernel (flushes, survivors flushed, flush cycles, deferrals, tiles). */
 int topk_debug_stats(uint64_t* host8, int reset) {
+    // (a variant build may compile only some select TUs with -DTOPK_DEBUG: the others
+    // have no counters and are skipped)
     for (int i = 0; i < 8; ++i) host8[i] = 0;
+    int found = 0;
     for (int i = 0; i < topk::kSelectTableN; ++i) {
         const auto f = topk::kSelectTable[i].debug;
-        if (f(topk::kDbgStatsAdd, host8, 0) != 0) return -1;
+        if (f(topk::kDbgStatsAdd, host8, 0) != 0) continue;
         if (reset && f(topk::kDbgStatsReset, nullptr, 0) != 0) return -1;
+        ++found;
     }
-    return 0;
+    return found ? 0 : -1;
 }
 
 topk_status_t topk_probe_read(const void* data, size_t bytes, int method, int grid, int tile,
