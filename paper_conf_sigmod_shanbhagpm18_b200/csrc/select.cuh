@@ -540,7 +540,7 @@ struct Ctx {
     int Lp;           // code network size log2 K' (K' = min(max(K, 16), 512)); -1: not used
     void* codes;      // shared: code-network scratch (8 x K' codes)
     bool filter;
-    bool boot;        // the kernel runs the boot sample (kBoot)
+    int boot_l2;      // kBoot: bag limit of the second flush (0: no boot sample)
 };
 
 // Sample rows in shared scratch: row r at scratch + r * ScrStride(G) (padded with zeros
@@ -775,10 +775,13 @@ __device__ int compact_bag(const SBuf<E>& buf, int cnt, E tau, int* s_w) {
 // cheap second flush soon publishes samples of many more keys (the boot samples cover
 // one buffer per CTA only) and the rank bound tightens early.  A stream flush always
 // leaves at most half of the next limit (progress: a warp appends <= 512 at a time).
-#ifndef TOPK_L2_BOOT
-#define TOPK_L2_BOOT 128
+#ifndef TOPK_L2_BOOT_MUL
+#define TOPK_L2_BOOT_MUL 4
 #endif
-__device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties, bool boot = false) {
+#ifndef TOPK_L2_BOOT_KMAX
+#define TOPK_L2_BOOT_KMAX 256
+#endif
+__device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties, int boot_l2 = 0) {
     // (K = 256: 512 measured 6 us faster than 1024, K = 128: 360 -> 354 us; other K: 512
     // no better, 2048 slower)
     const int l2 = (c_dbg >> 6) & 3 ? 512 * (1 + ((c_dbg >> 6) & 3))
@@ -790,9 +793,9 @@ __device__ __forceinline__ int next_limit(int nflush, int K, int Lp, int ties, b
     if (ties) return max(max(2 * K, K + 512), kCap >> 3);
     // After a boot sample (boot_sample) the bound already stands on a 16x larger sample:
     // the survivors arrive ~16x slower, so the second flush -- the one that publishes
-    // samples of many tiles -- comes at a much smaller bag.  (Progress: that flush makes
-    // nflush 2, whose limit is kCap.)
-    if (boot && nflush == 1 && Lp >= 0 && !(c_dbg & 4)) return TOPK_L2_BOOT;
+    // samples of many tiles -- comes at a much smaller bag (Ctx::boot_l2).  (Progress:
+    // that flush makes nflush 2, whose limit is kCap.)
+    if (boot_l2 > 0 && nflush == 1 && Lp >= 0 && !(c_dbg & 4)) return boot_l2;
     return (nflush == 1 && Lp >= 0 && !(c_dbg & 4)) ? max(l2, 2 * K) : kCap;
 }
 
@@ -861,7 +864,7 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         // (equal codes): finish exactly, and skip the code path from now on
         const bool weak = heavy || (cnt > 2 * K && 2 * cnt > cnt0);
         done = mode == kFlushStream && !weak &&
-               cnt <= next_limit(st->nflush + 1, K, cx.Lp, 0, cx.boot) / 2;
+               cnt <= next_limit(st->nflush + 1, K, cx.Lp, 0, cx.boot_l2) / 2;
         // (the boot sample's bag is emptied after this flush: no exact pass unless the
         // code bound was defeated by ties)
         if (st->req & kReqBoot) done = !weak;
@@ -914,7 +917,7 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         st->cnt_fail = 0x7FFFFFFF;
         st->sorted_cnt = done ? -1 : cnt;
         st->nflush += 1;
-        st->limit = next_limit(st->nflush, K, cx.Lp, st->ties, cx.boot);
+        st->limit = next_limit(st->nflush, K, cx.Lp, st->ties, cx.boot_l2);
         st->req = 0;
         trace(3);
     }
@@ -1365,7 +1368,14 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         cx.nrows = cx.J - cx.j_lo < maxrows ? cx.J - cx.j_lo : maxrows;
     }
     cx.filter = FILTER;
-    cx.boot = kBoot;
+    // Second flush after a boot sample (measured, 2^29 uniform): K <= 256 -- none (the
+    // boot bound is tight enough; k = 128 348 -> 338 us, k = 256 354 -> 352); larger K
+    // (the 480-entry boot bag has no k-th best) -- as soon as the bag holds 4x the
+    // deepest sample the stream rank bound uses (k = 1024: 64 entries, 391 -> 373 us;
+    // k = 2048: 128)
+    cx.boot_l2 = !kBoot ? 0
+                 : K <= TOPK_L2_BOOT_KMAX ? kCap
+                 : TOPK_L2_BOOT_MUL << (cx.j_lo + min(cx.nrows, TOPK_FLUSH_ROWS) - 1);
     // K > 512: the code network still gives the bag's 2^j-th best codes for j <= 9,
     // whose cross-CTA rank bound bounds the global k-th best (t = ceil(k / 2^j) <= G)
     cx.Lp = FILTER ? (K < 16 ? 4 : min(__ffs(K) - 1, 9)) : -1;
