@@ -69,6 +69,9 @@ namespace topk {
 #ifndef TOPK_BOOT_SMALL_K
 #define TOPK_BOOT_SMALL_K 256  // K from which the boot buffer is kCap / 8 entries (else kCap)
 #endif
+#ifndef TOPK_BOOT_WAIT_KMIN
+#define TOPK_BOOT_WAIT_KMIN 512  // K from which the boot flush waits for every CTA's samples
+#endif
 #ifndef TOPK_BOOT_SAMPLE
 #define TOPK_BOOT_SAMPLE 1  // boot bag = the best key of each consumer thread's share of tile 0
 #endif
@@ -80,6 +83,9 @@ namespace topk {
 #endif
 #ifndef TOPK_REFRESH_AT
 #define TOPK_REFRESH_AT 12  // tile index at which warp 0 requests a rank-bound refresh
+#endif
+#ifndef TOPK_REFRESH_AT_NOWAIT
+#define TOPK_REFRESH_AT_NOWAIT 6  // ... when the boot flush did not wait for its peers
 #endif
 
 constexpr int kNC = 480;                                    // consumer threads (15 warps)
@@ -541,6 +547,7 @@ struct Ctx {
     void* codes;      // shared: code-network scratch (8 x K' codes)
     bool filter;
     int boot_l2;      // kBoot: bag limit of the second flush (0: no boot sample)
+    bool boot_wait;   // the boot flush waits (<= 20 us) until every CTA published samples
 };
 
 // Sample rows in shared scratch: row r at scratch + r * ScrStride(G) (padded with zeros
@@ -695,7 +702,7 @@ __device__ void take_bounds(CtaState<typename KeyTraits<Key>::E, Key>* st, const
                             typename KeyTraits<Key>::E own, bool publish) {
     if (publish) {
         if (threadIdx.x == 0 && !own.is_sentinel()) tau_publish(cx.hdr, own);
-        if (!st->pubd && cx.G > 1 && !(c_dbg & 2)) {
+        if (cx.boot_wait && !st->pubd && cx.G > 1 && !(c_dbg & 2)) {
             // boot: every CTA flushes its first buffer at about the same time; wait for
             // their samples so the very first bound is the cross-CTA rank bound (a stale
             // or missing sample only weakens the bound -- the wait is a performance
@@ -725,6 +732,9 @@ __device__ void take_bounds(CtaState<typename KeyTraits<Key>::E, Key>* st, const
         if (!publish)
             for (int ji = 0; ji < kPubRows; ++ji) st->best[ji] = 0ull;
         if (cx.filter) fold_bounds<Key, MIN>(st, cx, own);
+        // (no boot wait: the first publishing flush still ends the boot; every read of
+        // pubd for this flush is behind us)
+        if (publish) st->pubd = 1;
     }
     CSync::sync();
 }
@@ -1353,6 +1363,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     const Key* keys = static_cast<const Key*>(p.keys);
     WsHeader* hdr = reinterpret_cast<WsHeader*>(p.ws);
     Ctx cx;
+    uint32_t refresh_at;  // tile index at which consumer thread 0 requests a rank-bound refresh
     cx.hdr = hdr;
     cx.pub = reinterpret_cast<unsigned long long*>(p.ws + ws_pub_offset());
     cx.scratch = scratch;
@@ -1373,6 +1384,11 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     // (the 480-entry boot bag has no k-th best) -- as soon as the bag holds 4x the
     // deepest sample the stream rank bound uses (k = 1024: 64 entries, 391 -> 373 us;
     // k = 2048: 128)
+    // Boot wait (measured with the boot sample): K <= 256 proceed on their own boot bound and
+    // pull the rank bound at tile 6 (k = 32 331 -> 328 us, k = 256 354 -> 352); larger K wait
+    // (without it k = 1024 375 -> 399 us) and refresh at tile 12
+    cx.boot_wait = !kBoot || K >= TOPK_BOOT_WAIT_KMIN;
+    refresh_at = cx.boot_wait ? TOPK_REFRESH_AT : TOPK_REFRESH_AT_NOWAIT;
     cx.boot_l2 = !kBoot ? 0
                  : K <= TOPK_L2_BOOT_KMAX ? kCap
                  : TOPK_L2_BOOT_MUL << (cx.j_lo + min(cx.nrows, TOPK_FLUSH_ROWS) - 1);
@@ -1591,7 +1607,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         __syncwarp();
         if (lane == 0) mbar_arrive(&empty[slot]);
         // Once every CTA has had time to publish its first run, pull the rank bound.
-        if (FILTER && G > 1 && tid == 0 && s == TOPK_REFRESH_AT) atomicOr(&st.req, kReqRefresh);
+        if (FILTER && G > 1 && tid == 0 && s == refresh_at) atomicOr(&st.req, kReqRefresh);
     }
     // Drain: serve requests of warps still streaming, until all are done.
     while (cbar_or(pending_req())) collective();
