@@ -383,7 +383,7 @@ struct CtaState {
     unsigned long long best[kPubRows];
     int npres[kPubRows];       // rank_rows: present samples per ranked row
     int nx;                    // kBoot, CTA 0: extras kept aside until the boot flush
-    unsigned long long xent[8];
+    E xent[8];
     uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
 };
 
@@ -412,6 +412,28 @@ __device__ __forceinline__ void bound_set(CtaState<E96, Key>* st, E96 t) {
         st->par = make_par<Key, MIN>(t);
     }
 }
+// Lower the bound by one entry step (the boot sample's re-read tile: keys >= the old bound
+// pass the strict test against the new one).  Thread 0 inside a collective.
+template <class Key, bool MIN>
+__device__ __forceinline__ void bound_weaken1(CtaState<E32, Key>* st) {
+    if (st->tau_w != 0ull) st->tau_w -= 1ull;
+}
+template <class Key, bool MIN>
+__device__ __forceinline__ void bound_weaken1(CtaState<E64, Key>* st) {
+    E64 t = st->tau;
+    if (t.is_sentinel()) return;
+    if (t.ni != 0u) {
+        t.ni -= 1u;
+    } else {
+        t.c -= 1ull;
+        t.ni = 0xFFFFFFFFu;
+    }
+    st->tau = t;
+    st->par = make_par<Key, MIN>(t);
+}
+template <class Key, bool MIN>
+__device__ __forceinline__ void bound_weaken1(CtaState<E96, Key>*) {}  // (no boot sample)
+
 // The bound a consumer uses for one tile (changes only inside collectives).
 template <class Key, bool MIN>
 __device__ __forceinline__ Par<E32, Key> load_par(const CtaState<E32, Key>& st) {
@@ -915,12 +937,12 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         TOPK_STAT(2, static_cast<unsigned long long>(clock64() - t0));
         if (!done) TOPK_STAT(6, 1ull);
         if (tried && !done && publish) st->ties = 1;
-        if constexpr (std::is_same<E, E32>::value) {
+        if constexpr (!std::is_same<E, E96>::value) {
             if (st->req & kReqBoot) {  // boot sample flushed (boot_sample): empty the bag
-                for (int q = 0; q < st->nx; ++q) buf.st(q, E32{st->xent[q]});  // (CTA 0)
+                for (int q = 0; q < st->nx; ++q) buf.st(q, st->xent[q]);  // (CTA 0)
                 cnt = st->nx;
                 done = true;
-                if (st->tau_w != 0ull) st->tau_w -= 1ull;  // keep >= the bound on re-read keys
+                bound_weaken1<Key, MIN>(st);  // keep >= the bound on re-read keys
             }
         }
         st->cnt = cnt;
@@ -962,22 +984,24 @@ __device__ void refresh(CtaState<typename KeyTraits<Key>::E, Key>* st, const Ctx
 // Collective (consumers); the bag is empty on entry.
 template <class Key, bool MIN>
 __device__ void boot_sample(const unsigned char* slot_data, uint32_t tlen, uint32_t lbase,
-                            const SBuf<E32>& buf, CtaState<E32, Key>* st) {
+                            const SBuf<typename KeyTraits<Key>::E>& buf,
+                            CtaState<typename KeyTraits<Key>::E, Key>* st) {
     using KT = KeyTraits<Key>;
+    using E = typename KT::E;
     constexpr int VEC = KT::kVec, ITEMS = Cfg<Key>::kItems;
     const Key* sk = reinterpret_cast<const Key*>(slot_data);
     const int tid = threadIdx.x;
-    E32 m = E32::sentinel();
+    E m = E::sentinel();
 #pragma unroll
     for (int q = 0; q < ITEMS; ++q) {
         const uint32_t pos = static_cast<uint32_t>((tid + (q / VEC) * kNC) * VEC + (q % VEC));
         if (pos < tlen) {
-            const E32 e = E32::make(KT::template code<MIN>(sk[pos]), lbase + pos);
+            const E e = E::make(KT::template code<MIN>(sk[pos]), lbase + pos);
             if (better(e, m)) m = e;
         }
     }
-    const E32 ents[1] = {m};
-    append<E32, 1>(buf, &st->cnt, ents, m.is_sentinel() ? 0u : 1u, kCap);  // <= kNC entries
+    const E ents[1] = {m};
+    append<E, 1>(buf, &st->cnt, ents, m.is_sentinel() ? 0u : 1u, kCap);  // <= kNC entries
     CSync::sync();
     if (threadIdx.x == 0) st->req |= kReqFlush | kReqBoot;  // flushed by the collective
     CSync::sync();
@@ -1336,11 +1360,12 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     constexpr int kStages = QC::kStages;
     constexpr int kSlot = QC::kSlotBytes;
     static_assert(Q == 0 || FILTER, "query forms run in filter mode");
-    // Boot sample (plain 32-bit-key form): the boot bag is the best key of each consumer
-    // thread's share of the first tile (480 entries, each the best of 16 keys) instead of
+    // Boot sample (plain form, f32 / u32 / f64 keys): the boot bag is the best key of each
+    // consumer thread's share of the first tile (480 entries, each the best of 16 -- f64: 8
+    // -- keys) instead of
     // the tile's first keys -- the same flush, a 16x larger sample behind its bound.  The
     // bag is then emptied and the tile consumed as usual.
-    constexpr bool kBoot = FILTER && Q == 0 && std::is_same<E, E32>::value && TOPK_BOOT_SAMPLE;
+    constexpr bool kBoot = FILTER && Q == 0 && !std::is_same<E, E96>::value && TOPK_BOOT_SAMPLE;
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ CtaState<E, Key> st;
@@ -1449,7 +1474,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
             if (tid < nextra) {
                 const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
                                                                      : tail0 + (tid - p.head);
-                st.xent[tid] = E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row)).v;
+                st.xent[tid] = E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row));
             }
             if (tid == 0) st.nx = nextra;
         } else {
@@ -1550,7 +1575,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                                   static_cast<uint32_t>(p.head + static_cast<uint64_t>(tile) * TK), buf, &st);
         } else {
             if (tid == 0) {
-                for (int q = 0; q < st.nx; ++q) buf.st(q, E32{st.xent[q]});
+                for (int q = 0; q < st.nx; ++q) buf.st(q, st.xent[q]);
                 st.cnt = st.nx;
             }
             CSync::sync();

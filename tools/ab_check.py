@@ -31,6 +31,10 @@ if os.environ.get("AB_CASES"):  # e.g. AB_CASES="29:uniform:1,256,1024;25:unifor
         CASES.append((1 << int(lg), dist, tuple(int(k) for k in ks.split(","))))
 
 
+DT = os.environ.get("AB_DTYPE", "f32")  # f32 | u32 | f64
+DC = {"f32": 0, "u32": 1, "f64": 2}[DT]
+
+
 def load(path):
     lib = ctypes.CDLL(path)
     vp, u64, u32, i32, sz = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int, ctypes.c_size_t
@@ -47,18 +51,18 @@ def main():
     handles = [load(p) for p in libs]
     st = torch.cuda.current_stream()
     for n, dist, ks in CASES:
-        x = datagen.generate(dist, n, "f32", seed=datagen.config_seed(2), device="cuda")
+        x = datagen.generate(dist, n, DT, seed=datagen.config_seed(2), device="cuda")
         keys = x.cpu().numpy()
         ov, oi = oracle.topk(keys, max(ks), True)
         for k in ks:
             for path, lib in zip(libs, handles):
-                ws = torch.zeros(int(lib.topk_workspace_bytes(0, n, k)), dtype=torch.uint8,
+                ws = torch.zeros(int(lib.topk_workspace_bytes(DC, n, k)), dtype=torch.uint8,
                                  device="cuda")
-                v = torch.empty(k, dtype=torch.float32, device="cuda")
+                v = torch.empty(k, dtype=x.dtype, device="cuda")
                 i = torch.empty(k, dtype=torch.int64, device="cuda")
 
                 def f():
-                    r = lib.topk_select(0, x.data_ptr(), None, n, 0, k, 0, 0, v.data_ptr(), None,
+                    r = lib.topk_select(DC, x.data_ptr(), None, n, 0, k, 0, 0, v.data_ptr(), None,
                                         i.data_ptr(), ws.data_ptr(), ws.numel(), st.cuda_stream)
                     assert r == 0, r
                 for _ in range(3):

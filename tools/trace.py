@@ -28,7 +28,8 @@ names = {1: "start", 2: "fb", 3: "fe", 4: "sEnd", 5: "tail", 6: "end", 7: "refr"
 for _e in range(32, 64): names[_e] = f"cnt{(_e - 32) * 64}+"
 send_c = [(max([t for e, t in ev if e == 4] or [0]), c) for c, ev in enumerate(rows)]
 send_c.sort()
-for _, c in send_c[:2] + send_c[-3:]:
+tail_c = [c for c, ev in enumerate(rows) if any(e == 5 for e, _ in ev)]
+for _, c in send_c[:2] + send_c[-2:] + [(0, c) for c in tail_c]:
     print(c, " ".join(f"{names[e]}@{(t - t0) / 1000:.1f}" for e, t in rows[c]))
 fl = [sum(1 for e, _ in ev if e == 2) for ev in rows]
 ft = []
