@@ -69,6 +69,9 @@ namespace topk {
 #ifndef TOPK_BOOT_SMALL_K
 #define TOPK_BOOT_SMALL_K 256  // K from which the boot buffer is kCap / 8 entries (else kCap)
 #endif
+#ifndef TOPK_BOOT_SAMPLE_Q
+#define TOPK_BOOT_SAMPLE_Q 1  // ... also for the query forms (rows passing the WHERE)
+#endif
 #ifndef TOPK_BOOT_WAIT_KMIN
 #define TOPK_BOOT_WAIT_KMIN 512  // K from which the boot flush waits for every CTA's samples
 #endif
@@ -1115,7 +1118,7 @@ __device__ __forceinline__ int consume_tile(const unsigned char* slot_data,
 // predicate -- "apply the filter predicate ... and then [write] it out into a shared
 // memory buffer" (FusedSortReducer), with the top-k bound as a second predicate.
 // Keys stay in registers (<= 8 per thread) for the exact test.
-template <class Key, bool MIN, int Q>
+template <class Key, bool MIN, int Q, bool SAMPLE = false>
 __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
                                               const Par<typename KeyTraits<Key>::E, Key>& pr,
                                               uint32_t tlen, uint32_t lbase,
@@ -1211,6 +1214,14 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
             for (int q = 0; q < ITEMS; ++q)
                 if (((mask >> q) & 1u) && !better(mk(q), pr.tau)) mask &= ~(1u << q);
         }
+        if constexpr (SAMPLE) {  // boot sample: the thread's best matching row only
+            E m = E::sentinel();
+#pragma unroll
+            for (int q = 0; q < ITEMS; ++q)
+                if (((mask >> q) & 1u) && better(mk(q), m)) m = mk(q);
+            const E one[1] = {m};
+            return append<E, 1>(buf, s_cnt, one, m.is_sentinel() ? 0u : 1u, limit);
+        }
         E ents[ITEMS];
 #pragma unroll
         for (int q = 0; q < ITEMS; ++q) ents[q] = mk(q);
@@ -1277,6 +1288,16 @@ __device__ __forceinline__ int consume_tile_q(const unsigned char* slot_data,
             if (((mask >> q) & 1u) &&
                 better(E::make(KT::template code<MIN>(x[q]), lbase + pos_of(q)), pr.tau))
                 keep |= 1u << q;
+    }
+    if constexpr (SAMPLE) {  // boot sample: the thread's best matching row only
+        E m = E::sentinel();
+#pragma unroll
+        for (int q = 0; q < ITEMS; ++q) {
+            const E e = E::make(KT::template code<MIN>(x[q]), lbase + pos_of(q));
+            if (((keep >> q) & 1u) && better(e, m)) m = e;
+        }
+        const E one[1] = {m};
+        return append<E, 1>(buf, s_cnt, one, m.is_sentinel() ? 0u : 1u, limit);
     }
     const int cnt = __popc(keep);
     int incl = cnt;
@@ -1365,7 +1386,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     // -- keys) instead of
     // the tile's first keys -- the same flush, a 16x larger sample behind its bound.  The
     // bag is then emptied and the tile consumed as usual.
-    constexpr bool kBoot = FILTER && Q == 0 && !std::is_same<E, E96>::value && TOPK_BOOT_SAMPLE;
+    constexpr bool kBoot = FILTER && !std::is_same<E, E96>::value && TOPK_BOOT_SAMPLE &&
+                           (Q == 0 || TOPK_BOOT_SAMPLE_Q);
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ CtaState<E, Key> st;
@@ -1471,12 +1493,21 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if constexpr (kBoot) {  // kept aside: the boot flush empties the bag, then adds them
             const uint64_t tail0 = p.head + p.body_n;
             const int nextra = static_cast<int>(p.head + (p.n - tail0));
-            if (tid < nextra) {
-                const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
-                                                                     : tail0 + (tid - p.head);
-                st.xent[tid] = E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row));
+            if constexpr (Q == 0) {
+                if (tid < nextra) {
+                    const uint64_t row = tid < static_cast<int>(p.head) ? static_cast<uint64_t>(tid)
+                                                                         : tail0 + (tid - p.head);
+                    st.xent[tid] = E::make(KT::template code<MIN>(keys[row]), static_cast<uint32_t>(row));
+                }
+                if (tid == 0) st.nx = nextra;
+            } else if (tid < 32) {  // query forms: head == 0, nextra <= 3; WHERE applies
+                const uint64_t row = tail0 + tid;
+                bool ok = tid < nextra;
+                if constexpr ((Q & kQPred) != 0) ok = ok && pred_ok(p, p.pred[ok ? row : 0]);
+                const uint32_t bal = __ballot_sync(0xFFFFFFFFu, ok);
+                if (ok) st.xent[__popc(bal & ((1u << tid) - 1u))] = query_entry<Key, MIN, Q>(p, keys, row);
+                if (tid == 0) st.nx = __popc(bal);
             }
-            if (tid == 0) st.nx = nextra;
         } else {
             append_extras();
         }
@@ -1570,9 +1601,18 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         if (lane == 0) tile = st.tile[0];
         tile = __shfl_sync(0xFFFFFFFFu, tile, 0);
         if (tile != kEndTile) {
-            boot_sample<Key, MIN>(ring, static_cast<uint32_t>(min(static_cast<uint64_t>(TK),
-                                                                  p.body_n - static_cast<uint64_t>(tile) * TK)),
-                                  static_cast<uint32_t>(p.head + static_cast<uint64_t>(tile) * TK), buf, &st);
+            const uint32_t tlen = static_cast<uint32_t>(
+                min(static_cast<uint64_t>(TK), p.body_n - static_cast<uint64_t>(tile) * TK));
+            const uint32_t lbase = static_cast<uint32_t>(p.head + static_cast<uint64_t>(tile) * TK);
+            if constexpr (Q == 0) {
+                boot_sample<Key, MIN>(ring, tlen, lbase, buf, &st);
+            } else {  // the thread's best row passing the WHERE, same entry as consume_tile_q
+                consume_tile_q<Key, MIN, Q, true>(ring, make_par<Key, MIN>(E::sentinel()), tlen,
+                                                  lbase, buf, &st.cnt, kCap, p);
+                CSync::sync();
+                if (tid == 0) st.req |= kReqFlush | kReqBoot;  // flushed by the collective
+                CSync::sync();
+            }
         } else {
             if (tid == 0) {
                 for (int q = 0; q < st.nx; ++q) buf.st(q, st.xent[q]);
