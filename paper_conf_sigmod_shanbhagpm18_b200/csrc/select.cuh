@@ -72,6 +72,9 @@ namespace topk {
 #ifndef TOPK_BOOT_SAMPLE_Q
 #define TOPK_BOOT_SAMPLE_Q 1  // ... also for the query forms (rows passing the WHERE)
 #endif
+#ifndef TOPK_BOOT_SAMPLE_E96
+#define TOPK_BOOT_SAMPLE_E96 1  // ... also for three compound keys (KKKV)
+#endif
 #ifndef TOPK_BOOT_WAIT_KMIN
 #define TOPK_BOOT_WAIT_KMIN 512  // K from which the boot flush waits for every CTA's samples
 #endif
@@ -435,7 +438,24 @@ __device__ __forceinline__ void bound_weaken1(CtaState<E64, Key>* st) {
     st->par = make_par<Key, MIN>(t);
 }
 template <class Key, bool MIN>
-__device__ __forceinline__ void bound_weaken1(CtaState<E96, Key>*) {}  // (no boot sample)
+__device__ __forceinline__ void bound_weaken1(CtaState<E96, Key>* st) {
+    E96 t = st->tau;
+    if (t.is_sentinel()) return;
+    // (c, c3, ni) lexicographic: subtract one from the 128-bit word with borrows
+    if (t.ni != 0u) {
+        t.ni -= 1u;
+    } else {
+        t.ni = 0xFFFFFFFFu;
+        if (t.c3 != 0u) {
+            t.c3 -= 1u;
+        } else {
+            t.c3 = 0xFFFFFFFFu;
+            t.c -= 1ull;
+        }
+    }
+    st->tau = t;
+    st->par = make_par<Key, MIN>(t);
+}
 
 // The bound a consumer uses for one tile (changes only inside collectives).
 template <class Key, bool MIN>
@@ -940,7 +960,7 @@ __device__ void flush(const SBuf<typename KeyTraits<Key>::E>& buf,
         TOPK_STAT(2, static_cast<unsigned long long>(clock64() - t0));
         if (!done) TOPK_STAT(6, 1ull);
         if (tried && !done && publish) st->ties = 1;
-        if constexpr (!std::is_same<E, E96>::value) {
+        {
             if (st->req & kReqBoot) {  // boot sample flushed (boot_sample): empty the bag
                 for (int q = 0; q < st->nx; ++q) buf.st(q, st->xent[q]);  // (CTA 0)
                 cnt = st->nx;
@@ -1386,8 +1406,8 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     // -- keys) instead of
     // the tile's first keys -- the same flush, a 16x larger sample behind its bound.  The
     // bag is then emptied and the tile consumed as usual.
-    constexpr bool kBoot = FILTER && !std::is_same<E, E96>::value && TOPK_BOOT_SAMPLE &&
-                           (Q == 0 || TOPK_BOOT_SAMPLE_Q);
+    constexpr bool kBoot = FILTER && TOPK_BOOT_SAMPLE && (Q == 0 || TOPK_BOOT_SAMPLE_Q) &&
+                           (!std::is_same<E, E96>::value || TOPK_BOOT_SAMPLE_E96);
 
     extern __shared__ __align__(128) unsigned char smem[];
     __shared__ CtaState<E, Key> st;
