@@ -269,3 +269,28 @@ def test_three_keys_full_ties_predicate_payload(cuda_device):
     col = u32col(N, 335, 10)
     pay = datagen.payload(N, seed=336)
     run_kkk(cols, 64, (False, False, True), pred=("range", col, 3, 8), payload=pay)
+
+
+@pytest.mark.parametrize("form", ["kk", "kkk", "rank", "pred"])
+def test_query_forms_repeated_calls_identical(form):
+    """The boot sample (select.cuh) runs in every query form: the first tile's best row per
+    thread is flushed, the bag emptied and the tile re-read against the bound weakened by
+    one entry step (E32 / E64 / E96 words).  The schedule is timing-dependent, the answer
+    must not be: 12 calls each, every one equal to the oracle."""
+    n = (1 << 22) + 4
+    a, b, c = (datagen.generate("uniform", n, "f32", seed=31 + j) for j in range(3))
+    col = u32col(n, 34)
+    ad, bd, cd, cold = a.cuda(), b.cuda(), c.cuda(), col.cuda()
+    if form == "kk":
+        f, exp = lambda: tk.topk_kk(ad, bd, 300)[2], oracle.topk_kk(host(a), host(b), 300)[2]
+    elif form == "kkk":
+        f = lambda: tk.topk_kkk(ad, bd, cd, 300)[3]
+        exp = oracle.topk_kkk(host(a), host(b), host(c), 300)[3]
+    elif form == "rank":
+        f = lambda: tk.query(ad, 300, True, rank_b=bd, rank_w=0.5)[1]
+        exp = oracle.query(host(a), 300, True, rank_b=host(b), rank_w=0.5)[1]
+    else:
+        f = lambda: tk.query(ad, 300, True, pred=("range", cold, 0, 1 << 31))[1]
+        exp = oracle.query(host(a), 300, True, pred=("range", host(col), 0, 1 << 31))[1]
+    bad = sum(int(not np.array_equal(f().cpu().numpy(), exp)) for _ in range(12))
+    assert bad == 0, f"{bad}/12 calls wrong"

@@ -45,5 +45,11 @@ col = datagen.generate("uniform", 1 << 20, "u32", seed=14)
 v, i = tk.query(xr.cuda(), 50, True, pred=("range", col.cuda(), 0, 1 << 31))
 ov, oi, m = oracle.query(xr.numpy(), 50, True, pred=("range", col.view(torch.int32).numpy().view(np.uint32), 0, 1 << 31))
 same(v, i, ov, oi)
+# compound keys (KKV: E64 entries, KKKV: E96 entries -- both run the boot sample)
+a, b, c = (datagen.generate("uniform", (1 << 20) + 4, "f32", seed=15 + j) for j in range(3))
+r = tk.topk_kk(a.cuda(), b.cuda(), 64)
+assert np.array_equal(r[2].cpu().numpy(), oracle.topk_kk(a.numpy(), b.numpy(), 64)[2])
+r = tk.topk_kkk(a.cuda(), b.cuda(), c.cuda(), 64)
+assert np.array_equal(r[3].cpu().numpy(), oracle.topk_kkk(a.numpy(), b.numpy(), c.numpy(), 64)[3])
 torch.cuda.synchronize()
 print("sanitize workload ok")
