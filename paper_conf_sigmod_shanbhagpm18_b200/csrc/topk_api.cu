@@ -322,6 +322,15 @@ static topk_status_t select_one(topk_dtype_t dtype, const void* keys, const uint
             return e ? static_cast<uint64_t>(std::strtoull(e, nullptr, 10)) : 0ull;
         }();
         uint64_t cap = static_cast<uint64_t>(sms);
+        // The merge tree above the CTAs costs a level per kPureGroup-fold of CTAs: up to
+        // 16 chunks run in ONE CTA (no tree: 2^12 keys, k = 32, graph-timed 11.9 -> 8.6
+        // us), up to 16 x 16 chunks in kPureGroup CTAs (one level); larger inputs spread
+        // over every SM (fewer busy warps per SM: faster chunks)
+        const uint64_t per_cta = static_cast<uint64_t>(topk::kPureNW);
+        if (nch <= per_cta)
+            cap = 1;
+        else if (nch <= per_cta * topk::kPureGroup && cap > static_cast<uint64_t>(topk::kPureGroup))
+            cap = topk::kPureGroup;
         if (grid_cap > 0 && grid_cap < cap) cap = grid_cap;
         const int pgrid = static_cast<int>(nch < cap ? nch : cap);
         const cudaError_t e = topk::launch_pure(key_kind(dtype), mn, pp, pgrid, st);
