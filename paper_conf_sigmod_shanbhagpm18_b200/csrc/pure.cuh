@@ -416,23 +416,29 @@ __global__ void __launch_bounds__(kPureNT, 1) pure_kernel(const PureParams p) {
         const int g0 = g * kPureGroup, gn = min(kPureGroup, G - g0);
         uint64_t* cand = p.cand;                           // G runs
         uint64_t* gcand = p.cand + static_cast<size_t>(G) * K;  // ng group runs
+        // (one gpu-scope fence, by the ticket thread after the barrier: cumulative over the
+        // run the CTA's threads stored before it; the last CTA's fence after the ticket
+        // orders the loads that follow the second barrier)
         for (int j = tid; j < K; j += kPureNT) __stcg(cand + blockIdx.x * K + j, b.ld(j).v);
-        __threadfence();
         __syncthreads();
-        if (tid == 0)
+        if (tid == 0) {
+            __threadfence();
             s_last = atomicAdd(p.ticket + 1 + g, 1u) == static_cast<unsigned>(gn - 1);
+            if (s_last) __threadfence();
+        }
         __syncthreads();
         if (!s_last) return;
-        __threadfence();
         merge_runs<L>(b, cand + static_cast<size_t>(g0) * K, gn, w, lane);
         if (ng > 1) {
             for (int j = tid; j < K; j += kPureNT) __stcg(gcand + g * K + j, b.ld(j).v);
-            __threadfence();
             __syncthreads();
-            if (tid == 0) s_last = atomicAdd(p.ticket, 1u) == static_cast<unsigned>(ng - 1);
+            if (tid == 0) {
+                __threadfence();
+                s_last = atomicAdd(p.ticket, 1u) == static_cast<unsigned>(ng - 1);
+                if (s_last) __threadfence();
+            }
             __syncthreads();
             if (!s_last) return;
-            __threadfence();
             merge_runs<L>(b, gcand, ng, w, lane);
         }
         if (tid <= ng) p.ticket[tid] = 0u;  // leave the workspace zeroed (all others done)
@@ -573,23 +579,29 @@ __global__ void __launch_bounds__(kPureNT, 1) pure64_kernel(const PureParams p) 
         const int g0 = g * kPureGroup, gn = min(kPureGroup, G - g0);
         uint64_t* cand = p.cand;
         uint64_t* gcand = p.cand + static_cast<size_t>(G) * K;
+        // (one gpu-scope fence, by the ticket thread after the barrier: cumulative over the
+        // run the CTA's threads stored before it; the last CTA's fence after the ticket
+        // orders the loads that follow the second barrier)
         for (int j = tid; j < K; j += kPureNT) __stcg(cand + blockIdx.x * K + j, b.ld(j).v);
-        __threadfence();
         __syncthreads();
-        if (tid == 0)
+        if (tid == 0) {
+            __threadfence();
             s_last = atomicAdd(p.ticket + 1 + g, 1u) == static_cast<unsigned>(gn - 1);
+            if (s_last) __threadfence();
+        }
         __syncthreads();
         if (!s_last) return;
-        __threadfence();
         merge_runs<L>(b, cand + static_cast<size_t>(g0) * K, gn, w, lane);
         if (ng > 1) {
             for (int j = tid; j < K; j += kPureNT) __stcg(gcand + g * K + j, b.ld(j).v);
-            __threadfence();
             __syncthreads();
-            if (tid == 0) s_last = atomicAdd(p.ticket, 1u) == static_cast<unsigned>(ng - 1);
+            if (tid == 0) {
+                __threadfence();
+                s_last = atomicAdd(p.ticket, 1u) == static_cast<unsigned>(ng - 1);
+                if (s_last) __threadfence();
+            }
             __syncthreads();
             if (!s_last) return;
-            __threadfence();
             merge_runs<L>(b, gcand, ng, w, lane);
         }
         if (tid <= ng) p.ticket[tid] = 0u;
