@@ -81,6 +81,9 @@ namespace topk {
 #ifndef TOPK_BOOT_SAMPLE
 #define TOPK_BOOT_SAMPLE 1  // boot bag = the best key of each consumer thread's share of tile 0
 #endif
+#ifndef TOPK_ADAPTIVE_ORDER
+#define TOPK_ADAPTIVE_ORDER 1
+#endif
 #ifndef TOPK_TAIL_ROWS
 #define TOPK_TAIL_ROWS 3
 #endif
@@ -388,6 +391,7 @@ struct CtaState {
     unsigned long long own_w;  // the bag's own k-th best as a bound word (0 = none)
     unsigned long long best[kPubRows];
     int npres[kPubRows];       // rank_rows: present samples per ranked row
+    int perm_mode;             // wave order: 0 undecided, 1 address order, 2 permuted
     int nx;                    // kBoot, CTA 0: extras kept aside until the boot flush
     E xent[8];
     uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
@@ -1472,6 +1476,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         fence_mbar_init();
         st.cnt = 0;
         st.nx = 0;
+        st.perm_mode = 0;
         st.cnt_fail = 0x7FFFFFFF;
         st.req = 0;
         st.nflush = 0;
@@ -1534,6 +1539,35 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
     }
     __syncthreads();
 
+    // Wave order (TOPK_ADAPTIVE_ORDER): waves after the first are visited in a pseudo-random
+    // order only if the input looks sorted -- 64 probe keys spread over it, >= 90 % of
+    // their neighbour pairs strictly increasing or strictly decreasing (every CTA probes
+    // the same keys, so every CTA takes the same decision).  A sorted input read in
+    // address order keeps raising the bound (every new wave beats all earlier ones: 2^29
+    // increasing, k = 256: 1064 us); any other input streams faster in address order
+    // (uniform 352 -> 345 us, few-distinct 369 -> 332, decreasing 360 -> 325).
+    if (tid < 32) {
+        const int lane0 = tid;
+        int mode = p.perm_h > 0 ? 2 : 1;
+        if constexpr (FILTER && Q == 0 && TOPK_ADAPTIVE_ORDER) {
+            if (p.perm_h > 0 && p.n >= 128) {
+                const uint64_t stp = p.n / 64;
+                const auto c0 = KT::template code<MIN>(keys[static_cast<uint64_t>(2 * lane0) * stp]);
+                const auto c1 = KT::template code<MIN>(keys[static_cast<uint64_t>(2 * lane0 + 1) * stp]);
+                const auto nx = __shfl_down_sync(0xFFFFFFFFu, c0, 1);
+                int inc = c1 > c0 ? 1 : 0, dec = c1 < c0 ? 1 : 0;
+                if (lane0 < 31) {
+                    inc += nx > c1 ? 1 : 0;
+                    dec += nx < c1 ? 1 : 0;
+                }
+                inc = __reduce_add_sync(0xFFFFFFFFu, inc);
+                dec = __reduce_add_sync(0xFFFFFFFFu, dec);
+                mode = (inc >= 57 || dec >= 57) ? 2 : 1;  // of 63 pairs
+            }
+        }
+        if (lane0 == 0) *reinterpret_cast<volatile int*>(&st.perm_mode) = mode;
+    }
+
     if (tid >= kNC) {
         // ---------------- producer warp (lane 0) ----------------
         if (tid != kNC) return;
@@ -1542,6 +1576,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
         const uint32_t blk = p.blk;
         const uint32_t nclaim = p.nwaves * p.wave * blk;
         uint32_t claim = 0, left = 0;
+        int mode = 0;  // wave order (st.perm_mode), read once
         uint32_t pending = atomicAdd(&hdr->next_tile, blk);
 #pragma unroll 1
         for (uint32_t s = 0;; ++s) {
@@ -1559,8 +1594,15 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                 // claim i -> block b = (wave, position); waves permuted, the blocks of a
                 // wave adjacent; tiles of a block in address order
                 const uint32_t b = i / blk;
-                const uint32_t pb =
-                    feistel_perm(b / p.wave, p.nwaves, p.perm_h) * p.wave + b % p.wave;
+                // address order, or the waves permuted (decided by the probe, which
+                // lands while the first claim's atomic is in flight)
+                const uint32_t wv = b / p.wave;
+                uint32_t pw = wv;
+                if (p.perm_h) {
+                    while (mode == 0) mode = *reinterpret_cast<volatile int*>(&st.perm_mode);
+                    if (mode == 2) pw = feistel_perm(wv, p.nwaves, p.perm_h);
+                }
+                const uint32_t pb = pw * p.wave + b % p.wave;
                 const uint32_t t = pb * blk + i % blk;
                 if (t < p.ntiles) {
                     tile = t;
