@@ -391,7 +391,7 @@ struct CtaState {
     unsigned long long own_w;  // the bag's own k-th best as a bound word (0 = none)
     unsigned long long best[kPubRows];
     int npres[kPubRows];       // rank_rows: present samples per ranked row
-    int perm_mode;             // wave order: 0 undecided, 1 address order, 2 permuted
+    int perm_mode;             // wave order: 0 undecided, 1 address, 2 permuted, 3 backwards
     int nx;                    // kBoot, CTA 0: extras kept aside until the boot flush
     E xent[8];
     uint32_t tile[kStagesMax];  // tile id of each ring slot (producer); kEndTile = done
@@ -1555,14 +1555,22 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                 const auto c0 = KT::template code<MIN>(keys[static_cast<uint64_t>(2 * lane0) * stp]);
                 const auto c1 = KT::template code<MIN>(keys[static_cast<uint64_t>(2 * lane0 + 1) * stp]);
                 const auto nx = __shfl_down_sync(0xFFFFFFFFu, c0, 1);
-                int inc = c1 > c0 ? 1 : 0, dec = c1 < c0 ? 1 : 0;
-                if (lane0 < 31) {
-                    inc += nx > c1 ? 1 : 0;
-                    dec += nx < c1 ? 1 : 0;
-                }
+                // signs of the 63 neighbour differences (probe j -> j + 1): d0 = c1 - c0,
+                // d1 = next lane's c0 - c1
+                const int s0 = c1 > c0 ? 1 : (c1 < c0 ? -1 : 0);
+                const int s1 = lane0 < 31 ? (nx > c1 ? 1 : (nx < c1 ? -1 : 0)) : 0;
+                const int sn = __shfl_down_sync(0xFFFFFFFFu, s0, 1);  // next lane's d0
+                int inc = (s0 > 0) + (s1 > 0), dec = (s0 < 0) + (s1 < 0);
+                // neighbouring differences of one sign: ~1/3 of the 62 for i.i.d. keys,
+                // nearly all for piecewise monotone input
+                int agree = (s0 != 0 && s0 == s1) + (lane0 < 31 && s1 != 0 && s1 == sn);
                 inc = __reduce_add_sync(0xFFFFFFFFu, inc);
                 dec = __reduce_add_sync(0xFFFFFFFFu, dec);
-                mode = (inc >= 57 || dec >= 57) ? 2 : 1;  // of 63 pairs
+                agree = __reduce_add_sync(0xFFFFFFFFu, agree);
+                // ascending codes (the best keys at the end): the waves backwards; descending
+                // codes (the best keys first): forwards; other piecewise monotone input (organ
+                // pipe, sawtooth): permuted; anything else: forwards
+                mode = inc >= 57 ? 3 : dec >= 57 ? 1 : agree >= 50 ? 2 : 1;
             }
         }
         if (lane0 == 0) *reinterpret_cast<volatile int*>(&st.perm_mode) = mode;
@@ -1601,6 +1609,7 @@ __global__ void __launch_bounds__(kNT, 1) select_kernel(const SelectParams p) {
                 if (p.perm_h) {
                     while (mode == 0) mode = *reinterpret_cast<volatile int*>(&st.perm_mode);
                     if (mode == 2) pw = feistel_perm(wv, p.nwaves, p.perm_h);
+                    if (mode == 3) pw = p.nwaves - 1u - wv;
                 }
                 const uint32_t pb = pw * p.wave + b % p.wave;
                 const uint32_t t = pb * blk + i % blk;
